@@ -1,0 +1,337 @@
+#!/usr/bin/env python3
+"""bench.py -- fundamental cycles balanced per second on B200 (BASELINE.json).
+
+One *step* = the whole hot path (roots + BFS +
+min-hash parents, Alg. 4 labels, Alg. 3 cycle traversal and balancing, flip
+and Harary-agree accumulation) over the workload's T trees per GPU; for N > 1
+ranks it also includes the NCCL all-reduce of the integer counters (L248).
+Trees are sharded t -> rank (t mod N), T per GPU (weak scaling).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c3] [--trees T]
+  python bench.py --impl reference ...   # the CPU oracle as the reference arm
+
+Prints ONE JSON line on rank 0.  Device time = CUDA events on the stream the
+library launches on, barrier + synchronize on both sides, max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+PAPER_BOOKS_CYCLES_PER_S = 12_294_896 / 0.8512   # PAPER.md L27, Table 3, Table 1
+METRIC = "fundamental cycles balanced/sec (device-timed)"
+DEFAULT_CONFIG = "c3"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default=DEFAULT_CONFIG)
+    ap.add_argument("--trees", type=int, default=0, help="trees per GPU per step (0 = config default)")
+    ap.add_argument("--walk", type=int, default=0)
+    ap.add_argument("--batch", type=int, default=0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample-trees", type=int, default=0)
+    return ap.parse_args()
+
+
+# ---------------------------------------------------------------------------
+# clocks during the timed region (B200_PROFILING.md)
+# ---------------------------------------------------------------------------
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.idx = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            p = [x.strip() for x in ln.split(",")]
+            if len(p) < 7:
+                continue
+            try:
+                sm.append(float(p[0]))
+                smax.append(float(p[1]))
+            except ValueError:
+                continue
+            for nm, val in zip(names, p[3:7]):
+                if val.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------------------
+# algorithmic byte model per tree: minimal compulsory
+# traffic of each phase, 4-byte ids / offsets
+# ---------------------------------------------------------------------------
+def phase_bytes(n, m, sumk, trees, batch):
+    words = (m + 31) // 32
+    return {
+        "init": 4 * n,                                   # dist reset
+        "bfs": 4 * (n + 1) + 24 * m + 12 * n,            # row_ptr, adj+eid+dist per slot, dist+key writes
+        "bottom_up": 32 * n,                             # key, edge, size RMW, parent/off writes
+        "top_down": 32 * n,                              # parent, parent label, offset, size; label writes
+        "cycles": 16 * m + 8 * (sumk / trees) + 4 * words,  # edge table, endpoint labels, k records, flip bits
+        "accumulate": 4 * words + (8 * m + 8 * n) / batch + 4 * n,
+    }
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+# ---------------------------------------------------------------------------
+def cpu_baseline(g, seed, trees, c_nt):
+    """The oracle as it stands (single-threaded C), on a bounded sample."""
+    import oracle
+    og = oracle.Graph.from_csr(g)
+    t0 = time.perf_counter()
+    og.balance(trees, seed)
+    dt = time.perf_counter() - t0
+    return {"value": trees * c_nt / dt, "unit": "cycles/s", "cores": 1, "kind": "oracle",
+            "sample": f"{trees} tree(s) of the same workload (seed {seed}), {dt:.2f} s, "
+                      f"single-threaded plain C (-O2)"}
+
+
+def sample_trees_for(g, requested):
+    if requested:
+        return requested
+    # ~10-30 s of oracle work: about 2e6 edges per tree-second on the host
+    return int(max(1, min(200, 4e7 / max(1, g.m))))
+
+
+def run_reference(args, g, desc, T):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    og = oracle.Graph.from_csr(g)
+    c_nt = g.m - g.n + og.ncomp
+    per_step = sample_trees_for(g, args.cpu_sample_trees)
+    for i in range(args.warmup):
+        og.balance(per_step, 1 + i, t_begin=0)
+    times = []
+    for s in range(args.steps):
+        t0 = time.perf_counter()
+        og.balance(per_step, 1000 + s)
+        times.append(time.perf_counter() - t0)
+    tot = sum(times)
+    val = args.steps * per_step * c_nt / tot
+    line = {
+        "impl": "reference", "metric": METRIC, "value": val, "unit": "cycles/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1000 * tot / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": val / PAPER_BOOKS_CYCLES_PER_S, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": f"{args.config}: {desc}", "n": g.n, "m": g.m,
+                   "trees_per_step": per_step, "note": "oracle = the reference arm of this tier"},
+        "cpu_baseline": {"value": val, "unit": "cycles/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{per_step} tree(s) per step of {args.config}"},
+        "e2e": {"value": val, "unit": "cycles/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    import graphgen
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    g, T_default, desc = graphgen.config(args.config)
+    T = args.trees or T_default
+    if args.impl == "reference":
+        return run_reference(args, g, desc, T)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_sc_alabanditrb21_b200 import graphb
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    graphb.set_option("walk", args.walk)
+    graphb.set_option("batch", args.batch)
+    graphb.load_graph(g)
+    n, m, ncomp = graphb.graph_info()
+    c_nt = m - n + ncomp
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream(dev)
+    cnt = torch.zeros(max(m, 1), dtype=torch.int32, device=dev)
+    agree = torch.zeros(n, dtype=torch.int32, device=dev)
+    total_trees = T * world
+
+    def step(seed):
+        graphb.balance_range(rank, total_trees, world, seed, cnt, agree, stream=stream)
+        if world > 1:
+            buf = torch.cat([cnt, agree])
+            dist.all_reduce(buf)
+
+    for i in range(args.warmup):
+        step(100 + i)
+    # per-phase CUDA events (library-internal, same stream) on one extra step
+    graphb.set_option("timing", 1)
+    step(99)
+    phase = graphb.stats()
+    graphb.set_option("timing", 0)
+
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clk = ClockSampler(local)
+    clk.start()
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    launches = 0
+    sumk = 0
+    ev0.record(stream)
+    for s in range(args.steps):
+        step(1 + s)
+        st = graphb.stats()
+        launches += st["launches"]
+        sumk += st["sum_cycle_len"]
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = clk.stop()
+    ms = ev0.elapsed_time(ev1)
+    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_max = float(t.item())
+    cycles_total = args.steps * total_trees * c_nt
+    value = cycles_total / (ms_max / 1000.0)
+
+    # roofline of the dominant phase (from the timed-phase step)
+    ph = phase["phase_ms"]
+    dom = max(ph, key=lambda k: ph[k])
+    per_tree_sumk = phase["sum_cycle_len"] / max(1, phase["trees"])
+    bytes_per_tree = phase_bytes(n, m, per_tree_sumk * phase["trees"], phase["trees"], phase["batch"])
+    trees_in_step = phase["trees"]
+    launches_of = {"cycles": max(1, phase["batches"] * -(-phase["batch"] // max(1, phase["cycle_group"])))}
+    dom_launches = launches_of.get(dom, phase["batches"])
+    dom_bytes_per_launch = bytes_per_tree[dom] * trees_in_step / dom_launches
+    dom_ms_per_launch = ph[dom] / dom_launches
+    peak, peak_src = load_peaks()
+    achieved = dom_bytes_per_launch / (dom_ms_per_launch / 1000.0) / 1e9
+    roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+                "bytes_per_launch": dom_bytes_per_launch, "launch_ms": dom_ms_per_launch,
+                "phase_share": {k: v / max(1e-9, sum(ph.values())) for k, v in ph.items()}}
+
+    # end-to-end through the public API with host buffers (rank-local)
+    e2e = None
+    if not args.no_e2e:
+        pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory().numpy()
+        hrp, hcol, hsg = pin(g.row_ptr), pin(g.col), pin(g.sign)
+        h_cnt = torch.empty(max(m, 1), dtype=torch.int32).pin_memory()
+        h_agr = torch.empty(n, dtype=torch.int32).pin_memory()
+        e_steps = max(1, min(args.steps, 3))
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for s in range(e_steps):
+            graphb.load_csr(hrp, hcol, hsg)
+            cnt.zero_(); agree.zero_()
+            step(500 + s)
+            h_cnt.copy_(cnt); h_agr.copy_(agree)
+            torch.cuda.synchronize()
+        el = time.perf_counter() - t0
+        tt = torch.tensor([el], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        e2e = {"value": e_steps * total_trees * c_nt / float(tt.item()), "unit": "cycles/s",
+               "h2d_bytes_per_step": int(hrp.nbytes + hcol.nbytes + hsg.nbytes),
+               "d2h_bytes_per_step": int(4 * (m + n)),
+               "note": "per step: gb_load_csr (H2D + ingest) + balance + D2H of the counters"}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(g, 1, sample_trees_for(g, args.cpu_sample_trees), c_nt)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "cycles/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
+            "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": value / PAPER_BOOKS_CYCLES_PER_S,
+            "vs_baseline_ref": "paper: 14.44M cycles/s, Amazon Books, Titan V (L27, L395) -- context",
+            "dtype": "u32", "data": "synthetic",
+            "config": {"workload": f"{args.config}: {desc}", "n": n, "m": m, "components": ncomp,
+                       "cycles_per_tree": c_nt, "trees_per_gpu": T, "trees_total": total_trees,
+                       "batch": phase["batch"], "cycle_group": phase["cycle_group"],
+                       "walk": "two-ended" if args.walk == 0 else "alg3-descent",
+                       "avg_cycle_len": per_tree_sumk / max(1, c_nt),
+                       "max_depth": phase["max_depth"],
+                       "l2": "inputs larger than L2 (graph arrays > 126 MB)" if 16 * m > 126e6
+                             else "graph fits L2; consecutive steps use new seeds (new trees)",
+                       "parallelism": f"trees t mod {world}; NCCL all-reduce of counters" if world > 1
+                                      else "1 GPU"},
+            "gpu_launches": launches,
+            "phase_ms_per_step": {k: v for k, v in ph.items()},
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "clocks": clocks,
+        }
+        print(json.dumps(line), flush=True)
+    graphb.free()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,141 @@
+/* graphb.h -- C ABI of the B200-native graphB+ balancing hot path.
+ *
+ * What it computes (PAPER.md = /root/reference/PAPER.md, Alabandi et al.,
+ * "Discovering and Balancing Fundamental Cycles in Large Signed Graphs", SC'21):
+ *
+ *   Alg. 2 (L125-L138): for k sampled spanning trees T of Sigma (method M =
+ *     BFS, L116-L123, "random BFS trees" L479), find the nearest balanced state
+ *     Sigma_T (Alg. 1 L96-L108, computed the graphB+ way, Alg. 3 L176-L202 with
+ *     the labels of Alg. 4) and form its Harary bipartition (L224);
+ *   L144: status(v) = (1/|T|) sum_T delta_T(v), delta = 1 / 0.5 / 0;
+ *   L248: count per vertex over the trees and reduce.
+ *
+ * Outputs are integer counters over the trees:
+ *   edge_flip_counts[e] = #trees in which the sign of undirected edge e is
+ *                         switched (Alg. 1; tree edges never are),
+ *   vertex_agree[v]     = sum_T 2*delta_T(v) (half-units: 2 larger Harary side,
+ *                         1 tie, 0 smaller side), so status(v) = agree/(2T).
+ *
+ * Conventions:
+ *   - m counts undirected edges; the CSR has 2m slots (Table 1, R2).
+ *   - eid(u,v) = rank of (min(u,v), max(u,v)) in lexicographic order.
+ *   - The tree of index t is defined by (graph, seed, t) only: root of
+ *     component C = C's vertices (ascending) [rkey(seed,t,C) mod |C|]; BFS
+ *     distances; parent(w) = neighbour one level up whose edge has the
+ *     minimum ekey(seed,t,eid) (R4).  Disconnected inputs are forests (R3).
+ *   - A non-tree edge gets the sign that makes its fundamental cycle even
+ *     (L214): flip(e) = (#negative tree edges on the path + neg(e)) mod 2 (R1).
+ *
+ * All calls return GB_OK (0) or a negative gb_err and set gb_last_error().
+ * Not thread-safe; one loaded graph per process, on the CUDA device current at
+ * gb_load_csr time.  Every step runs in the library's sm_100a kernels; there
+ * is no CPU fallback: without a usable CUDA device calls return GB_ECUDA.
+ */
+#ifndef GRAPHB_H
+#define GRAPHB_H
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum gb_err {
+    GB_OK = 0,
+    GB_EINVAL = -1, /* invalid argument or input graph                     */
+    GB_ESTATE = -2, /* no graph loaded                                     */
+    GB_ENOMEM = -3, /* device or host allocation failed                    */
+    GB_ECUDA = -4   /* CUDA runtime error (message in gb_last_error)       */
+};
+
+/* Load a signed graph Sigma = (G, sigma) (one compact
+ * CSR, allocated once).  Host arrays, borrowed for the call and copied:
+ *   row_ptr [n+1] int64, row_ptr[0] = 0, non-decreasing, row_ptr[n] = 2m
+ *   col_idx [2m]  int32, each row strictly increasing (sorted, no duplicates),
+ *                 no self loops, 0 <= col < n
+ *   sign    [2m]  int8, each +1 or -1, sign(u,v) == sign(v,u) (symmetric)
+ * Limits: 1 <= n < 2^31, 2m < 2^32.  Returns GB_EINVAL on any violation (also
+ * NULL pointers with m > 0).  A second call replaces the loaded graph. */
+int gb_load_csr(int64_t n, int64_t m, const int64_t *row_ptr,
+                const int32_t *col_idx, const int8_t *sign);
+
+/* Alg. 2 over trees t = 0 .. num_trees-1 (0 <= num_trees <= 2^30-1).
+ * Host outputs, caller-allocated, written in full on success, untouched on
+ * error: out_edge_flip_counts [m] indexed by eid, out_vertex_agree [n].
+ * num_trees == 0 writes zeros. */
+int gb_balance(int64_t num_trees, uint64_t seed,
+               uint32_t *out_edge_flip_counts, uint32_t *out_vertex_agree);
+
+/* Release all device and host state.  Idempotent. */
+void gb_free(void);
+
+/* ---- extensions (sharding, tests, measurement) -------------------------- */
+
+/* Trees t_begin, t_begin+t_stride, ... < t_end (the tree sharding of L248).
+ * DEVICE outputs on the loaded graph's device, ACCUMULATED (+=):
+ *   d_edge_cnt [m] int32, d_vertex_agree [n] int32.
+ * cuda_stream: a cudaStream_t to run on (NULL = the library's own stream).
+ * Asynchronous with respect to the host when cuda_stream is given. */
+int gb_balance_range(int64_t t_begin, int64_t t_end, int64_t t_stride, uint64_t seed,
+                     int32_t *d_edge_cnt, int32_t *d_vertex_agree, void *cuda_stream);
+
+/* One tree, every stage copied back to host arrays (any pointer may be NULL):
+ *   parent[n] (-1 at roots), dist[n] (BFS level), pre[n] (pre-order ID,
+ *   Alg. 3 step 1; any valid pre-order of T -- sibling order is not fixed,
+ *   R5), size[n] (subtree size, Alg. 4), flip[m] (0/1 by eid),
+ *   sum_cycle_len (sum over non-tree edges of the fundamental-cycle length,
+ *   counting e itself; L230), num_cycles (= m - n + #components, L112). */
+int gb_tree_debug(int64_t t, uint64_t seed, int32_t *parent, int32_t *dist,
+                  int32_t *pre, int32_t *size, uint8_t *flip,
+                  uint64_t *sum_cycle_len, int64_t *num_cycles);
+
+/* Alg. 3 on a caller tree (host parent[n], -1 at roots): returns flip[m] and
+ * the cycle statistics.  GB_EINVAL unless parent is a spanning forest of the
+ * loaded graph with exactly one root per connected component. */
+int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
+                          uint64_t *sum_cycle_len, int64_t *num_cycles);
+
+/* Options (before gb_balance*): "batch" trees per batch (0 = auto),
+ * "cycle_group" trees per cycle-kernel pass (0 = auto), "walk"
+ * (0 = two-ended interval walk, 1 = Alg. 3 descent with warp ballots),
+ * "timing" (1 = record per-phase CUDA events), "graphs" (1 = CUDA graphs). */
+int gb_set_option(const char *key, int64_t value);
+
+/* Statistics of the last gb_balance / gb_balance_range call:
+ * ints[0] trees, [1] sum of cycle lengths, [2] cycles, [3] kernel launches,
+ * [4] batches, [5] max tree depth, [6] batch size used, [7] cycle group used.
+ * phase_ms[GB_NPHASE] (valid when "timing" was 1): summed CUDA-event times.
+ * Returns the number of ints written. */
+#define GB_NPHASE 6
+#define GB_PHASE_INIT 0   /* roots, workspace reset                      */
+#define GB_PHASE_BFS 1    /* level-synchronous BFS + min-hash parents    */
+#define GB_PHASE_UP 2     /* Alg. 4 bottom-up sizes (+ sibling offsets)  */
+#define GB_PHASE_DOWN 3   /* Alg. 4 top-down pre-order IDs + ranges + pi */
+#define GB_PHASE_CYCLE 4  /* Alg. 3 cycle traversal + balancing          */
+#define GB_PHASE_ACCUM 5  /* counter accumulation + Harary agree         */
+int gb_get_stats(int64_t *ints, int n_ints, double *phase_ms, int n_phase);
+
+/* Per-tree statistics of the last gb_balance* call, for at most max_trees
+ * trees in processing order: out[3*i] = sum of cycle lengths, out[3*i+1] =
+ * cycles, out[3*i+2] = depth; tree_ids[i] = t.  Returns the count. */
+int64_t gb_tree_stats(uint64_t *out, int64_t *tree_ids, int64_t max_trees);
+
+/* Ingest results (§8 a.1), copied to host arrays (any pointer may be NULL):
+ * edge_u[m], edge_v[m] (u < v), edge_neg[m] (1 = negative) indexed by eid;
+ * slot_eid[2m] (eid of every CSR slot); comp[n] (component rank, components
+ * ordered by their minimum vertex). */
+int gb_graph_debug(int32_t *edge_u, int32_t *edge_v, int8_t *edge_neg,
+                   uint32_t *slot_eid, int32_t *comp);
+
+/* Loaded graph: n, m, number of connected components. */
+int gb_graph_info(int64_t *n, int64_t *m, int64_t *ncomp);
+
+/* Host-only self test of the library's hash (no GPU needed): SplitMix64
+ * vector and the inverse used to decode parent keys.  0 = pass. */
+int gb_selftest(void);
+
+const char *gb_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

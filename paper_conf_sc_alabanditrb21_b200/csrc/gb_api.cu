@@ -1,0 +1,512 @@
+// gb_api.cu -- the C ABI (include/graphb.h) and host orchestration: device
+// state owned from gb_load_csr to gb_free, per-batch workspaces allocated
+// once (L236: "all required dynamic memory is allocated once"), batches of B
+// trees driven asynchronously on one stream (§8 a.9), per-phase CUDA events
+// (Fig. 11 L451-L467 breakdown), counters accumulated on the device and
+// copied back once.
+#include "gb_internal.cuh"
+#include "../../include/graphb.h"
+
+#include <algorithm>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+namespace gb {
+
+static std::string g_err;
+void set_error(const std::string &msg) { g_err = msg; }
+
+struct Options {
+    int64_t batch = 0;       // 0 = auto
+    int64_t cycle_group = 0; // 0 = auto
+    int64_t walk = 0;        // 0 two-ended, 1 Alg. 3 descent
+    int64_t timing = 0;
+};
+
+struct Stats {
+    int64_t trees = 0, launches = 0, batches = 0, batch_used = 0, group_used = 0;
+    uint64_t sumk = 0, cycles = 0;
+    int64_t max_depth = 0;
+    double phase_ms[GB_NPHASE] = {0};
+    std::vector<uint64_t> per_tree;   // 3 per recorded tree
+    std::vector<int64_t> tree_ids;
+};
+
+struct State {
+    bool loaded = false;
+    Graph g;
+    Workspace ws;
+    bool ws_descent = false;
+    cudaStream_t stream = nullptr;
+    int32_t *d_cnt = nullptr, *d_agree = nullptr;  // gb_balance's device counters
+    int32_t *d_given = nullptr;                    // caller tree (gb_balance_given_tree)
+    unsigned long long *d_visited = nullptr;       // [kMaxBatch]
+    unsigned long long *d_rec_stats = nullptr;     // [kRecCap][3]
+    std::vector<int32_t> h_comp;
+    Options opt;
+    Stats st;
+};
+static State S;
+constexpr int64_t kRecCap = 1 << 16;  // per-tree statistics kept for gb_tree_stats
+
+static void free_ws(Workspace &w) {
+    void *ptrs[] = {w.dist, w.pkey, w.sz, w.qv, w.qs, w.lvl, w.vbase, w.pinfo, w.peid,
+                    w.off, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth, w.tstat, w.maxd,
+                    w.cidx, w.cstart, w.clist, w.crec, w.scan_tmp};
+    for (void *p : ptrs) if (p) cudaFree(p);
+    w = Workspace();
+}
+
+static void free_graph(Graph &g) {
+    void *ptrs[] = {g.row_ptr, g.adj, g.adj_eid, g.edges, g.comp, g.coff, g.cverts};
+    for (void *p : ptrs) if (p) cudaFree(p);
+    g = Graph();
+}
+
+static size_t per_tree_bytes(const Graph &g, bool descent) {
+    const size_t n = (size_t)g.n;
+    size_t b = 64 * n + 12 * 2 + 4 * (size_t)((g.m + 31) / 32) + 4 * (size_t)g.ncomp;
+    if (descent) b += 20 * n;
+    return b;
+}
+
+#define ALLOC(ptr, count)                                                            \
+    do {                                                                             \
+        cudaError_t _e = cudaMalloc((void **)&(ptr), sizeof(*(ptr)) * (size_t)std::max<int64_t>(count, 1)); \
+        if (_e != cudaSuccess) {                                                     \
+            set_error(std::string("cudaMalloc " #ptr ": ") + cudaGetErrorString(_e)); \
+            free_ws(S.ws);                                                           \
+            return _e == cudaErrorMemoryAllocation ? GB_ENOMEM : GB_ECUDA;           \
+        }                                                                            \
+    } while (0)
+
+static int ensure_workspace(int B, bool descent) {
+    if (S.ws.B >= B && (!descent || S.ws_descent)) return GB_OK;
+    B = std::max(B, S.ws.B);
+    descent = descent || S.ws_descent;
+    free_ws(S.ws);
+    Workspace &w = S.ws;
+    const Graph &g = S.g;
+    const int64_t n = g.n, Bn = (int64_t)B * n, words = (g.m + 31) / 32;
+    ALLOC(w.dist, Bn);
+    ALLOC(w.pkey, Bn);
+    ALLOC(w.sz, Bn);
+    ALLOC(w.qv, Bn);
+    ALLOC(w.qs, Bn);
+    ALLOC(w.lvl, (int64_t)B * (n + 2));
+    ALLOC(w.vbase, (int64_t)B * (n + 2));
+    ALLOC(w.pinfo, Bn);
+    ALLOC(w.peid, Bn);
+    ALLOC(w.off, Bn);
+    ALLOC(w.pp, Bn);
+    ALLOC(w.rec, Bn);
+    ALLOC(w.fbits, (int64_t)B * words);
+    ALLOC(w.s1, (int64_t)B * g.ncomp);
+    ALLOC(w.tkey, kMaxBatch);
+    ALLOC(w.depth, kMaxBatch);
+    ALLOC(w.tstat, 2 * kMaxBatch);
+    ALLOC(w.maxd, 1);
+    if (descent) {
+        ALLOC(w.cidx, Bn);
+        ALLOC(w.cstart, Bn);
+        ALLOC(w.clist, Bn);
+        ALLOC(w.crec, Bn);
+        w.scan_tmp_elems = scan_tmp_elems(Bn);
+        ALLOC(w.scan_tmp, (int64_t)w.scan_tmp_elems);
+    }
+    w.B = B;
+    w.n = n;
+    S.ws_descent = descent;
+    return GB_OK;
+}
+
+static int check_device() {
+    int dev = -1;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) {
+        set_error(std::string("no usable CUDA device: ") + cudaGetErrorString(e));
+        return GB_ECUDA;
+    }
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev < 1) {
+        set_error("no CUDA device");
+        return GB_ECUDA;
+    }
+    return GB_OK;
+}
+
+// ---------------------------------------------------------------------------
+// small device helpers
+// ---------------------------------------------------------------------------
+__global__ void k_tree_keys(uint64_t *tkey, int B, uint64_t seed, int64_t t0, int64_t stride) {
+    int b = threadIdx.x;
+    if (b < B) tkey[b] = tree_key(seed, t0 + (int64_t)b * stride);
+}
+
+__global__ void k_record_stats(const unsigned long long *tstat, const int32_t *depth, int B,
+                               unsigned long long *rec, int64_t pos, int64_t cap) {
+    int b = threadIdx.x;
+    if (b < B && pos + b < cap) {
+        rec[3 * (pos + b)] = tstat[2 * b];
+        rec[3 * (pos + b) + 1] = tstat[2 * b + 1];
+        rec[3 * (pos + b) + 2] = (unsigned long long)depth[b];
+    }
+}
+
+static int auto_batch(int64_t ntrees) {
+    if (S.opt.batch > 0) return (int)std::min<int64_t>(S.opt.batch, kMaxBatch);
+    size_t freeb = 0, totb = 0;
+    cudaMemGetInfo(&freeb, &totb);
+    size_t have = freeb + (size_t)S.ws.B * per_tree_bytes(S.g, S.ws_descent);
+    int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk == 1));
+    int64_t b = std::min<int64_t>({ntrees, (int64_t)kMaxBatch, std::max<int64_t>(bm, 1)});
+    // large graphs: a few trees per batch already fill the GPU
+    if (S.g.n >= (1 << 22)) b = std::min<int64_t>(b, 8);
+    return (int)std::max<int64_t>(b, 1);
+}
+
+static int auto_group(int B) {
+    if (S.opt.cycle_group > 0) return (int)std::min<int64_t>(S.opt.cycle_group, B);
+    // keep the labels of the trees walked together L2-resident (~48 MB)
+    double per = 12.0 * (double)S.g.n;
+    int g = (int)std::max(1.0, std::floor(48.0e6 / per));
+    return std::max(1, std::min(g, B));
+}
+
+// the whole hot path over trees t_begin, t_begin+stride, ... < t_end
+static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_t seed,
+                         int32_t *d_cnt, int32_t *d_agree, cudaStream_t st) {
+    Stats &T = S.st;
+    T = Stats();
+    const int64_t K = t_end > t_begin ? (t_end - t_begin + stride - 1) / stride : 0;
+    if (K == 0) return GB_OK;
+    const bool descent = S.opt.walk == 1;
+    if (descent && (int64_t)kMaxBatch * S.g.n >= (1ll << 32)) {
+        set_error("walk=1 needs batch*n < 2^32");
+        return GB_EINVAL;
+    }
+    const int B = auto_batch(K);
+    int rc = ensure_workspace(B, descent);
+    if (rc) return rc;
+    const int G = auto_group(B);
+    T.batch_used = B;
+    T.group_used = G;
+    if (!S.d_rec_stats) {
+        GB_CUDA_TRY(cudaMalloc(&S.d_rec_stats, sizeof(unsigned long long) * 3 * kRecCap));
+    }
+    std::vector<cudaEvent_t> evs;
+    const bool timing = S.opt.timing != 0;
+    int64_t done = 0;
+    while (done < K) {
+        const int nb = (int)std::min<int64_t>(B, K - done);
+        const int64_t t0 = t_begin + done * stride;
+        cudaEvent_t *ev = nullptr;
+        if (timing) {
+            size_t base = evs.size();
+            evs.resize(base + GB_NPHASE + 1);
+            for (int i = 0; i <= GB_NPHASE; i++) cudaEventCreate(&evs[base + i]);
+            ev = evs.data() + base;
+        }
+        k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, nb, seed, t0, stride);
+        ++T.launches;
+        GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 2 * nb, st));
+        rc = run_batch_tree(S.g, S.ws, nb, nullptr, nullptr, st, &T.launches, ev, descent);
+        if (rc) return rc;
+        if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
+        rc = run_batch_cycles(S.g, S.ws, nb, G, descent, st, &T.launches);
+        if (rc) return rc;
+        if (ev) GB_CUDA_TRY(cudaEventRecord(ev[5], st));
+        rc = run_batch_accumulate(S.g, S.ws, nb, d_cnt, d_agree, st, &T.launches);
+        if (rc) return rc;
+        if (ev) GB_CUDA_TRY(cudaEventRecord(ev[6], st));
+        if (done < kRecCap) {
+            k_record_stats<<<1, kMaxBatch, 0, st>>>(S.ws.tstat, S.ws.depth, nb, S.d_rec_stats, done, kRecCap);
+            ++T.launches;
+            for (int b = 0; b < nb && done + b < kRecCap; b++) T.tree_ids.push_back(t0 + b * stride);
+        }
+        done += nb;
+        T.batches++;
+    }
+    GB_CUDA_TRY(cudaGetLastError());
+    const int64_t nrec = std::min<int64_t>(K, kRecCap);
+    T.per_tree.resize(3 * nrec);
+    GB_CUDA_TRY(cudaMemcpyAsync(T.per_tree.data(), S.d_rec_stats, sizeof(uint64_t) * 3 * nrec,
+                                cudaMemcpyDeviceToHost, st));
+    GB_CUDA_TRY(cudaStreamSynchronize(st));
+    T.trees = K;
+    for (int64_t i = 0; i < nrec; i++) {
+        T.sumk += T.per_tree[3 * i];
+        T.cycles += T.per_tree[3 * i + 1];
+        T.max_depth = std::max<int64_t>(T.max_depth, (int64_t)T.per_tree[3 * i + 2]);
+    }
+    if (timing) {
+        for (size_t base = 0; base < evs.size(); base += GB_NPHASE + 1) {
+            for (int i = 0; i < GB_NPHASE; i++) {
+                float ms = 0;
+                cudaEventElapsedTime(&ms, evs[base + i], evs[base + i + 1]);
+                T.phase_ms[i] += ms;
+            }
+        }
+        for (auto e : evs) cudaEventDestroy(e);
+    }
+    return GB_OK;
+}
+
+static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
+    Stats &T = S.st;
+    T = Stats();
+    int rc = ensure_workspace(1, S.opt.walk == 1);
+    if (rc) return rc;
+    cudaStream_t st = S.stream;
+    k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, 1, seed, t, 1);
+    ++T.launches;
+    GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 2, st));
+    rc = run_batch_tree(S.g, S.ws, 1, nullptr, d_given, st, &T.launches, nullptr, S.opt.walk == 1);
+    if (rc) return rc;
+    if (d_given) {
+        unsigned long long vis = 0;
+        GB_CUDA_TRY(cudaMemcpyAsync(&vis, S.ws.tstat, sizeof(vis), cudaMemcpyDeviceToHost, st));
+        GB_CUDA_TRY(cudaStreamSynchronize(st));
+        if ((int64_t)vis != S.g.n) {
+            set_error("parent is not a spanning forest of the loaded graph (some vertex is not "
+                      "reachable from a root through parent edges)");
+            return GB_EINVAL;
+        }
+        GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 2, st));
+    }
+    rc = run_batch_cycles(S.g, S.ws, 1, 1, S.opt.walk == 1, st, &T.launches);
+    if (rc) return rc;
+    GB_CUDA_TRY(cudaStreamSynchronize(st));
+    return GB_OK;
+}
+
+static int copy_flips(uint8_t *flip) {
+    const int64_t words = (S.g.m + 31) / 32;
+    std::vector<uint32_t> fb(std::max<int64_t>(words, 1));
+    if (words) GB_CUDA_TRY(cudaMemcpy(fb.data(), S.ws.fbits, 4 * words, cudaMemcpyDeviceToHost));
+    for (int64_t e = 0; e < S.g.m; e++) flip[e] = (fb[e >> 5] >> (e & 31)) & 1u;
+    return GB_OK;
+}
+
+static int copy_cycle_stats(uint64_t *sumk, int64_t *ncyc) {
+    unsigned long long ts[2] = {0, 0};
+    GB_CUDA_TRY(cudaMemcpy(ts, S.ws.tstat, sizeof(ts), cudaMemcpyDeviceToHost));
+    if (sumk) *sumk = ts[0];
+    if (ncyc) *ncyc = (int64_t)ts[1];
+    return GB_OK;
+}
+
+}  // namespace gb
+
+using namespace gb;
+
+extern "C" {
+
+const char *gb_last_error(void) { return g_err.c_str(); }
+
+int gb_selftest(void) {
+    // SplitMix64 public vector from state 0
+    const uint64_t kat[3] = {0xE220A8397B1DCDAFull, 0x6E789E6AA1B965F4ull, 0x06C45D188009454Full};
+    for (int i = 0; i < 3; i++)
+        if (tree_key(0, i) != kat[i]) { set_error("selftest: SplitMix64 vector"); return GB_EINVAL; }
+    uint64_t x = 0x0123456789ABCDEFull;
+    for (int i = 0; i < 100000; i++) {
+        x = x * 6364136223846793005ull + 1442695040888963407ull;
+        if (unmix64(mix64(x)) != x) { set_error("selftest: unmix64"); return GB_EINVAL; }
+        uint32_t e = (uint32_t)(x >> 33);
+        if (edge_of_key(x, edge_key(x, e)) != e) { set_error("selftest: edge key decode"); return GB_EINVAL; }
+    }
+    return GB_OK;
+}
+
+void gb_free(void) {
+    if (S.loaded || S.ws.B) {
+        free_ws(S.ws);
+        free_graph(S.g);
+    }
+    if (S.d_cnt) cudaFree(S.d_cnt);
+    if (S.d_agree) cudaFree(S.d_agree);
+    if (S.d_given) cudaFree(S.d_given);
+    if (S.d_visited) cudaFree(S.d_visited);
+    if (S.d_rec_stats) cudaFree(S.d_rec_stats);
+    if (S.stream) cudaStreamDestroy(S.stream);
+    Options keep = S.opt;
+    S = State();
+    S.opt = keep;
+}
+
+int gb_load_csr(int64_t n, int64_t m, const int64_t *row_ptr, const int32_t *col_idx,
+                const int8_t *sign) {
+    if (n < 1 || n >= (1ll << 31)) { set_error("n must satisfy 1 <= n < 2^31"); return GB_EINVAL; }
+    if (m < 0 || 2 * m >= (1ll << 32)) { set_error("m must satisfy 0 <= 2m < 2^32"); return GB_EINVAL; }
+    if (!row_ptr || (m > 0 && (!col_idx || !sign))) { set_error("NULL input array"); return GB_EINVAL; }
+    if (row_ptr[0] != 0 || row_ptr[n] != 2 * m) {
+        set_error("row_ptr[0] must be 0 and row_ptr[n] must equal 2m");
+        return GB_EINVAL;
+    }
+    int rc = check_device();
+    if (rc) return rc;
+    gb_free();
+    int dev = 0;
+    GB_CUDA_TRY(cudaGetDevice(&dev));
+    int coop = 0;
+    GB_CUDA_TRY(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev));
+    if (!coop) { set_error("device lacks cooperative launch"); return GB_ECUDA; }
+    S.g.dev = dev;
+    GB_CUDA_TRY(cudaDeviceGetAttribute(&S.g.num_sms, cudaDevAttrMultiProcessorCount, dev));
+    GB_CUDA_TRY(cudaStreamCreateWithFlags(&S.stream, cudaStreamNonBlocking));
+    int64_t launches = 0;
+    rc = ingest(S.g, n, m, row_ptr, col_idx, sign, S.stream, &launches);
+    if (rc) { gb_free(); return rc; }
+    S.h_comp.resize(n);
+    GB_CUDA_TRY(cudaMemcpy(S.h_comp.data(), S.g.comp, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+    S.loaded = true;
+    S.st = Stats();
+    S.st.launches = launches;
+    return GB_OK;
+}
+
+int gb_graph_debug(int32_t *edge_u, int32_t *edge_v, int8_t *edge_neg, uint32_t *slot_eid,
+                   int32_t *comp) {
+    if (!S.loaded) { set_error("no graph loaded"); return GB_ESTATE; }
+    const int64_t m = S.g.m, n = S.g.n;
+    if (m && (edge_u || edge_v || edge_neg)) {
+        std::vector<uint2> e(m);
+        GB_CUDA_TRY(cudaMemcpy(e.data(), S.g.edges, sizeof(uint2) * m, cudaMemcpyDeviceToHost));
+        for (int64_t i = 0; i < m; i++) {
+            if (edge_u) edge_u[i] = (int32_t)e[i].x;
+            if (edge_v) edge_v[i] = (int32_t)(e[i].y & kIdMask);
+            if (edge_neg) edge_neg[i] = (int8_t)(e[i].y >> 31);
+        }
+    }
+    if (m && slot_eid)
+        GB_CUDA_TRY(cudaMemcpy(slot_eid, S.g.adj_eid, sizeof(uint32_t) * 2 * m, cudaMemcpyDeviceToHost));
+    if (comp) GB_CUDA_TRY(cudaMemcpy(comp, S.g.comp, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+    return GB_OK;
+}
+
+int gb_graph_info(int64_t *n, int64_t *m, int64_t *ncomp) {
+    if (!S.loaded) { set_error("no graph loaded"); return GB_ESTATE; }
+    if (n) *n = S.g.n;
+    if (m) *m = S.g.m;
+    if (ncomp) *ncomp = S.g.ncomp;
+    return GB_OK;
+}
+
+int gb_set_option(const char *key, int64_t value) {
+    if (!key) { set_error("NULL option"); return GB_EINVAL; }
+    if (!strcmp(key, "batch")) { if (value < 0) return GB_EINVAL; S.opt.batch = value; }
+    else if (!strcmp(key, "cycle_group")) { if (value < 0) return GB_EINVAL; S.opt.cycle_group = value; }
+    else if (!strcmp(key, "walk")) { if (value != 0 && value != 1) return GB_EINVAL; S.opt.walk = value; }
+    else if (!strcmp(key, "timing")) S.opt.timing = value != 0;
+    else if (!strcmp(key, "graphs")) { /* reserved */ }
+    else { set_error(std::string("unknown option ") + key); return GB_EINVAL; }
+    return GB_OK;
+}
+
+int gb_balance_range(int64_t t_begin, int64_t t_end, int64_t t_stride, uint64_t seed,
+                     int32_t *d_edge_cnt, int32_t *d_vertex_agree, void *cuda_stream) {
+    if (!S.loaded) { set_error("no graph loaded"); return GB_ESTATE; }
+    if (t_begin < 0 || t_end < t_begin || t_stride < 1 || t_end > (1ll << 30) - 1) {
+        set_error("bad tree range");
+        return GB_EINVAL;
+    }
+    if ((S.g.m > 0 && !d_edge_cnt) || !d_vertex_agree) { set_error("NULL output"); return GB_EINVAL; }
+    cudaStream_t st = cuda_stream ? (cudaStream_t)cuda_stream : S.stream;
+    return balance_range(t_begin, t_end, t_stride, seed, d_edge_cnt, d_vertex_agree, st);
+}
+
+int gb_balance(int64_t num_trees, uint64_t seed, uint32_t *out_edge_flip_counts,
+               uint32_t *out_vertex_agree) {
+    if (!S.loaded) { set_error("no graph loaded"); return GB_ESTATE; }
+    if (num_trees < 0 || num_trees > (1ll << 30) - 1) { set_error("num_trees out of range"); return GB_EINVAL; }
+    if ((S.g.m > 0 && !out_edge_flip_counts) || !out_vertex_agree) { set_error("NULL output"); return GB_EINVAL; }
+    if (!S.d_cnt) {
+        GB_CUDA_TRY(cudaMalloc(&S.d_cnt, sizeof(int32_t) * std::max<int64_t>(S.g.m, 1)));
+        GB_CUDA_TRY(cudaMalloc(&S.d_agree, sizeof(int32_t) * S.g.n));
+    }
+    GB_CUDA_TRY(cudaMemsetAsync(S.d_cnt, 0, sizeof(int32_t) * std::max<int64_t>(S.g.m, 1), S.stream));
+    GB_CUDA_TRY(cudaMemsetAsync(S.d_agree, 0, sizeof(int32_t) * S.g.n, S.stream));
+    int rc = balance_range(0, num_trees, 1, seed, S.d_cnt, S.d_agree, S.stream);
+    if (rc) return rc;
+    if (S.g.m)
+        GB_CUDA_TRY(cudaMemcpyAsync(out_edge_flip_counts, S.d_cnt, sizeof(int32_t) * S.g.m,
+                                    cudaMemcpyDeviceToHost, S.stream));
+    GB_CUDA_TRY(cudaMemcpyAsync(out_vertex_agree, S.d_agree, sizeof(int32_t) * S.g.n,
+                                cudaMemcpyDeviceToHost, S.stream));
+    GB_CUDA_TRY(cudaStreamSynchronize(S.stream));
+    return GB_OK;
+}
+
+int gb_tree_debug(int64_t t, uint64_t seed, int32_t *parent, int32_t *dist, int32_t *pre,
+                  int32_t *size, uint8_t *flip, uint64_t *sum_cycle_len, int64_t *num_cycles) {
+    if (!S.loaded) { set_error("no graph loaded"); return GB_ESTATE; }
+    if (t < 0 || t > (1ll << 30) - 1) { set_error("bad tree index"); return GB_EINVAL; }
+    int rc = run_single_tree(t, seed, nullptr);
+    if (rc) return rc;
+    const int64_t n = S.g.n;
+    std::vector<uint32_t> tmp(n);
+    if (parent) {
+        GB_CUDA_TRY(cudaMemcpy(tmp.data(), S.ws.pinfo, 4 * n, cudaMemcpyDeviceToHost));
+        for (int64_t v = 0; v < n; v++) parent[v] = tmp[v] == kNone ? -1 : (int32_t)(tmp[v] & kIdMask);
+    }
+    if (dist) GB_CUDA_TRY(cudaMemcpy(dist, S.ws.dist, 4 * n, cudaMemcpyDeviceToHost));
+    if (pre) {
+        GB_CUDA_TRY(cudaMemcpy(tmp.data(), S.ws.pp, 4 * n, cudaMemcpyDeviceToHost));
+        for (int64_t v = 0; v < n; v++) pre[v] = (int32_t)(tmp[v] & kIdMask);
+    }
+    if (size) {
+        std::vector<unsigned long long> s64(n);
+        GB_CUDA_TRY(cudaMemcpy(s64.data(), S.ws.sz, 8 * n, cudaMemcpyDeviceToHost));
+        for (int64_t v = 0; v < n; v++) size[v] = (int32_t)(uint32_t)s64[v];
+    }
+    if (flip) { rc = copy_flips(flip); if (rc) return rc; }
+    return copy_cycle_stats(sum_cycle_len, num_cycles);
+}
+
+int gb_balance_given_tree(const int32_t *parent, uint8_t *flip, uint64_t *sum_cycle_len,
+                          int64_t *num_cycles) {
+    if (!S.loaded) { set_error("no graph loaded"); return GB_ESTATE; }
+    if (!parent) { set_error("NULL parent"); return GB_EINVAL; }
+    const int64_t n = S.g.n;
+    std::vector<int32_t> roots(S.g.ncomp, 0);
+    for (int64_t v = 0; v < n; v++) {
+        if (parent[v] == -1) roots[S.h_comp[v]]++;
+        else if (parent[v] < 0 || parent[v] >= n || parent[v] == v) {
+            set_error("parent entry out of range");
+            return GB_EINVAL;
+        }
+    }
+    for (int64_t c = 0; c < S.g.ncomp; c++)
+        if (roots[c] != 1) { set_error("need exactly one root (-1) per connected component"); return GB_EINVAL; }
+    if (!S.d_given) GB_CUDA_TRY(cudaMalloc(&S.d_given, sizeof(int32_t) * n));
+    GB_CUDA_TRY(cudaMemcpy(S.d_given, parent, sizeof(int32_t) * n, cudaMemcpyHostToDevice));
+    int rc = run_single_tree(0, 0, S.d_given);
+    if (rc) return rc;
+    if (flip) { rc = copy_flips(flip); if (rc) return rc; }
+    return copy_cycle_stats(sum_cycle_len, num_cycles);
+}
+
+int gb_get_stats(int64_t *ints, int n_ints, double *phase_ms, int n_phase) {
+    const Stats &T = S.st;
+    int64_t v[8] = {T.trees, (int64_t)T.sumk, (int64_t)T.cycles, T.launches, T.batches,
+                    T.max_depth, T.batch_used, T.group_used};
+    int k = 0;
+    for (; ints && k < n_ints && k < 8; k++) ints[k] = v[k];
+    for (int i = 0; phase_ms && i < n_phase && i < GB_NPHASE; i++) phase_ms[i] = T.phase_ms[i];
+    return k;
+}
+
+int64_t gb_tree_stats(uint64_t *out, int64_t *tree_ids, int64_t max_trees) {
+    const Stats &T = S.st;
+    int64_t k = std::min<int64_t>(max_trees, (int64_t)T.tree_ids.size());
+    for (int64_t i = 0; i < k; i++) {
+        if (out) for (int j = 0; j < 3; j++) out[3 * i + j] = T.per_tree[3 * i + j];
+        if (tree_ids) tree_ids[i] = T.tree_ids[i];
+    }
+    return k;
+}
+
+}  // extern "C"

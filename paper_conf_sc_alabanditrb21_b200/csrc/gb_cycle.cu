@@ -1,0 +1,294 @@
+// gb_cycle.cu -- §8 rows a.6-a.8:
+//   a.6 cycle traversal + balancing (Alg. 3),
+//   a.7 Harary majority and per-vertex agree (L144, L224, L248),
+//   a.8 accumulation without contended atomics.
+//
+// Cycle walk.  The labels of Alg. 4 make "x is an ancestor of y" an interval
+// test: pre x <= pre y <= pre x + size x - 1 (L212: the range of the edge
+// into x).  Two walks are provided; both traverse every edge of the
+// fundamental cycle exactly once, XOR its negative bits and count its length:
+//
+//  walk 0 (two-ended, §8 f.1): one thread per non-tree edge (u,v).  u climbs
+//   while it is not an ancestor of v, v climbs while it is not an ancestor of
+//   u; both stop at the LCA.  Each step is one 8-byte gather of the
+//   pre-indexed record {parent pre | neg, size}; the two climbs are
+//   independent, so every thread keeps two loads in flight.
+//  walk 1 (Alg. 3 as written, §8 a.6): u climbs to the LCA through parent
+//   edges (the inverse range of L212), then the warp descends from the LCA to
+//   v: at each vertex the child whose range contains pre v is found with a
+//   coalesced load of up to 32 sorted child starts and one __ballot_sync
+//   (32-ary pivot rounds for hubs), L214.
+//
+// Either way: c = XOR of the negative tree edges; the non-tree edge gets the
+// sign (-1)^c, i.e. flip = c XOR neg(e) (reading R1).  No synchronization is
+// needed: the tree is read-only and every non-tree edge has one writer (L309).
+#include "gb_internal.cuh"
+#include "../../include/graphb.h"
+
+#include <algorithm>
+
+namespace gb {
+
+struct CycleParams {
+    const uint2 *edges;
+    int64_t n, m;
+    const uint32_t *pp;    // [B][n] pre | pi<<31
+    const uint2 *rec;      // [B][n] pre-indexed {up | neg<<31, size}
+    const uint2 *crec;     // [B][n] pre-indexed {child-list start, #children}
+    const uint32_t *clist; // children pre IDs, per parent ascending
+    uint32_t *fbits;       // [B][words]
+    unsigned long long *tstat;  // [B][2]
+    int64_t words;
+    int b0, G;             // trees b0 .. b0+G-1 of the batch
+};
+
+constexpr int kCycleBlock = 256;
+constexpr int kMaxGroup = 64;
+
+__device__ __forceinline__ bool is_anc(uint32_t a, uint32_t size_a, uint32_t t) {
+    return (t - a) < size_a;  // a <= t <= a + size_a - 1 (unsigned wrap for t < a)
+}
+
+// one warp = 32 consecutive edges (one flip word per tree)
+__global__ void __launch_bounds__(kCycleBlock) k_cycles_two_ended(CycleParams P) {
+    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup];
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; }
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t word = gw; word < P.words; word += nw) {
+        const int64_t e = word * 32 + lane;
+        const bool valid = e < P.m;
+        uint2 ed = valid ? __ldg(P.edges + e) : make_uint2(0, 0);
+        const uint32_t u = ed.x, v = ed.y & kIdMask, nege = ed.y >> 31;
+        for (int g = 0; g < P.G; g++) {
+            const size_t nb = (size_t)(P.b0 + g) * P.n;
+            const uint2 *rec = P.rec + nb;
+            uint32_t flip = 0, k = 0;
+            bool cyc = false;
+            if (valid) {
+                const uint32_t x0 = __ldg(P.pp + nb + u) & kIdMask;
+                const uint32_t y0 = __ldg(P.pp + nb + v) & kIdMask;
+                uint2 rx = __ldg(rec + x0), ry = __ldg(rec + y0);
+                // tree edge iff one endpoint is the other's parent (simple graph)
+                if ((rx.x & kIdMask) != y0 && (ry.x & kIdMask) != x0) {
+                    cyc = true;
+                    uint32_t x = x0, y = y0, c = 0;
+                    k = 1;
+                    bool ax = is_anc(x, rx.y, y0), ay = is_anc(y, ry.y, x0);
+                    while (!(ax && ay)) {
+                        if (!ax) {
+                            c ^= rx.x;
+                            x = rx.x & kIdMask;
+                            rx = __ldg(rec + x);
+                            k++;
+                            ax = is_anc(x, rx.y, y0);
+                        }
+                        if (!ay) {
+                            c ^= ry.x;
+                            y = ry.x & kIdMask;
+                            ry = __ldg(rec + y);
+                            k++;
+                            ay = is_anc(y, ry.y, x0);
+                        }
+                    }
+                    flip = (c >> 31) ^ nege;
+                }
+            }
+            const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
+            if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
+            // per-tree cycle statistics (warp reduce, then shared atomics)
+            uint32_t kk = k, cc = cyc ? 1u : 0u;
+#pragma unroll
+            for (int d = 16; d; d >>= 1) {
+                kk += __shfl_xor_sync(0xFFFFFFFFu, kk, d);
+                cc += __shfl_xor_sync(0xFFFFFFFFu, cc, d);
+            }
+            if (lane == 0 && cc) {
+                atomicAdd(&s_k[g], (unsigned long long)kk);
+                atomicAdd(&s_c[g], (unsigned long long)cc);
+            }
+        }
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) {
+        if (s_c[i]) {
+            atomicAdd(P.tstat + 2 * (P.b0 + i), s_k[i]);
+            atomicAdd(P.tstat + 2 * (P.b0 + i) + 1, s_c[i]);
+        }
+    }
+}
+
+// Alg. 3 as written: lane-parallel climb to the LCA, then warp-cooperative
+// descents from the LCA to v, one lane's cycle at a time.
+__global__ void __launch_bounds__(kCycleBlock) k_cycles_descent(CycleParams P) {
+    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup];
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; }
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t word = gw; word < P.words; word += nw) {
+        const int64_t e = word * 32 + lane;
+        const bool valid = e < P.m;
+        uint2 ed = valid ? __ldg(P.edges + e) : make_uint2(0, 0);
+        const uint32_t u = ed.x, v = ed.y & kIdMask, nege = ed.y >> 31;
+        for (int g = 0; g < P.G; g++) {
+            const size_t nb = (size_t)(P.b0 + g) * P.n;
+            const uint2 *rec = P.rec + nb;
+            const uint2 *crec = P.crec + nb;
+            uint32_t c = 0, k = 0, x = 0, y0 = 0;
+            bool cyc = false;
+            if (valid) {
+                const uint32_t x0 = __ldg(P.pp + nb + u) & kIdMask;
+                y0 = __ldg(P.pp + nb + v) & kIdMask;
+                uint2 rx = __ldg(rec + x0), ry = __ldg(rec + y0);
+                if ((rx.x & kIdMask) != y0 && (ry.x & kIdMask) != x0) {
+                    cyc = true;
+                    k = 1;
+                    x = x0;
+                    // the parent edge's range is the complement of x's range
+                    // (L212): follow it while pre v is outside x's range
+                    while (!is_anc(x, rx.y, y0)) {
+                        c ^= rx.x;
+                        x = rx.x & kIdMask;
+                        rx = __ldg(rec + x);
+                        k++;
+                    }
+                }
+            }
+            // descents: the whole warp serves one lane's cycle at a time
+            uint32_t pending = __ballot_sync(0xFFFFFFFFu, cyc && x != y0);
+            while (pending) {
+                const int src = __ffs(pending) - 1;
+                pending &= pending - 1;
+                uint32_t cx = __shfl_sync(0xFFFFFFFFu, x, src);
+                const uint32_t ty = __shfl_sync(0xFFFFFFFFu, y0, src);
+                uint32_t cpar = 0, steps = 0;
+                while (cx != ty) {
+                    // children of cx: clist[cs .. cs+nc), ascending pre; find
+                    // the last child start <= ty (its range holds ty)
+                    const uint2 cr = __ldg(crec + cx);
+                    uint32_t lo = cr.x, cnt = cr.y;
+                    while (cnt > 32) {
+                        const uint32_t step = (cnt + 31) >> 5;
+                        const uint32_t pos = lane * step;
+                        const uint32_t pv = pos < cnt ? __ldg(P.clist + lo + pos) : 0xFFFFFFFFu;
+                        const uint32_t bal = __ballot_sync(0xFFFFFFFFu, pv <= ty);
+                        const uint32_t h = 31 - __clz(bal);
+                        const uint32_t nlo = h * step;
+                        cnt = min(step, cnt - nlo);
+                        lo += nlo;
+                    }
+                    const uint32_t cv = lane < cnt ? __ldg(P.clist + lo + lane) : 0xFFFFFFFFu;
+                    const uint32_t bal = __ballot_sync(0xFFFFFFFFu, cv <= ty);
+                    const uint32_t ch = __shfl_sync(0xFFFFFFFFu, cv, 31 - __clz(bal));
+                    cpar ^= __ldg(rec + ch).x;   // neg bit of the edge into ch
+                    cx = ch;
+                    steps++;
+                }
+                if (lane == src) { c ^= cpar; k += steps; }
+            }
+            const uint32_t flip = cyc ? ((c >> 31) ^ nege) : 0u;
+            const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
+            if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
+            uint32_t kk = k, cc = cyc ? 1u : 0u;
+#pragma unroll
+            for (int d = 16; d; d >>= 1) {
+                kk += __shfl_xor_sync(0xFFFFFFFFu, kk, d);
+                cc += __shfl_xor_sync(0xFFFFFFFFu, cc, d);
+            }
+            if (lane == 0 && cc) {
+                atomicAdd(&s_k[g], (unsigned long long)kk);
+                atomicAdd(&s_c[g], (unsigned long long)cc);
+            }
+        }
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) {
+        if (s_c[i]) {
+            atomicAdd(P.tstat + 2 * (P.b0 + i), s_k[i]);
+            atomicAdd(P.tstat + 2 * (P.b0 + i) + 1, s_c[i]);
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// a.8: per batch, edge_cnt[e] += sum_b flip_b(e) (one coalesced RMW per edge
+// per batch; the B flip words of a 32-edge group are warp-broadcast loads)
+// and a.7: agree[v] += sum_b 2*delta_b(v), delta from the root-parity sides:
+// side(v) = pi(v); per component s1 = #{pi = 1}, s0 = |C| - s1 (L144, L224).
+// ---------------------------------------------------------------------------
+__global__ void k_accumulate_edges(const uint32_t *__restrict__ fbits, int64_t words, int64_t m,
+                                   int B, int32_t *__restrict__ cnt) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t w = e >> 5;
+        const uint32_t sh = (uint32_t)(e & 31);
+        int32_t s = 0;
+        for (int b = 0; b < B; b++) s += (__ldg(fbits + (size_t)b * words + w) >> sh) & 1u;
+        if (s) cnt[e] += s;
+    }
+}
+
+__global__ void k_accumulate_agree(const uint32_t *__restrict__ pp, const uint32_t *__restrict__ s1,
+                                   const int32_t *__restrict__ comp, const int32_t *__restrict__ coff,
+                                   int64_t n, int64_t ncomp, int B, int32_t *__restrict__ agree) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t C = __ldg(comp + v);
+        const uint32_t cs = (uint32_t)(__ldg(coff + C + 1) - __ldg(coff + C));
+        int32_t d = 0;
+        for (int b = 0; b < B; b++) {
+            const uint32_t ones = __ldg(s1 + (size_t)b * ncomp + C);
+            const uint32_t mine = (__ldg(pp + (size_t)b * n + v) >> 31) ? ones : cs - ones;
+            const uint32_t other = cs - mine;
+            d += mine > other ? 2 : (mine == other ? 1 : 0);
+        }
+        agree[v] += d;
+    }
+}
+
+static unsigned grid_cap(int64_t work, int threads, int sms, int per_sm) {
+    int64_t b = (work + threads - 1) / threads;
+    int64_t cap = (int64_t)sms * per_sm;
+    return (unsigned)std::max<int64_t>(1, std::min(b, cap));
+}
+
+int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool descent,
+                     cudaStream_t st, int64_t *launches) {
+    CycleParams P;
+    P.edges = g.edges; P.n = g.n; P.m = g.m;
+    P.pp = ws.pp; P.rec = ws.rec; P.crec = ws.crec; P.clist = ws.clist;
+    P.fbits = ws.fbits; P.tstat = ws.tstat;
+    P.words = (g.m + 31) / 32;
+    if (P.words == 0) return GB_OK;
+    group = std::max(1, std::min(group, kMaxGroup));
+    for (int b0 = 0; b0 < B; b0 += group) {
+        P.b0 = b0;
+        P.G = std::min(group, B - b0);
+        unsigned grid = grid_cap(P.words * 32, kCycleBlock, g.num_sms, 8);
+        if (descent) k_cycles_descent<<<grid, kCycleBlock, 0, st>>>(P);
+        else k_cycles_two_ended<<<grid, kCycleBlock, 0, st>>>(P);
+        ++*launches;
+    }
+    GB_CUDA_TRY(cudaGetLastError());
+    return GB_OK;
+}
+
+int run_batch_accumulate(const Graph &g, Workspace &ws, int B, int32_t *d_cnt, int32_t *d_agree,
+                         cudaStream_t st, int64_t *launches) {
+    const int64_t words = (g.m + 31) / 32;
+    if (g.m) {
+        k_accumulate_edges<<<grid_cap(g.m, 256, g.num_sms, 16), 256, 0, st>>>(ws.fbits, words, g.m, B, d_cnt);
+        ++*launches;
+    }
+    k_accumulate_agree<<<grid_cap(g.n, 256, g.num_sms, 16), 256, 0, st>>>(
+        ws.pp, ws.s1, g.comp, g.coff, g.n, g.ncomp, B, d_agree);
+    ++*launches;
+    GB_CUDA_TRY(cudaGetLastError());
+    return GB_OK;
+}
+
+}  // namespace gb

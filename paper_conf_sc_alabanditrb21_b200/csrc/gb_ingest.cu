@@ -1,0 +1,400 @@
+// gb_ingest.cu -- §8 row a.1: CSR ingest with per-edge ids (once per load).
+//
+// one compact CSR holds Sigma; L238: 1-bit sign flags packed
+// next to the 31-bit ids; L333: the paper keeps only the LCC -- here forests
+// are accepted (reading R3), so connected components are labelled once.
+//
+// Everything runs on the device: validation (sorted simple symmetric rows,
+// signs +-1 and symmetric), edge ids eid(u,v) = rank of (min,max) (the rank
+// of an upper slot is ebase[u] + its position among row u's upper slots),
+// packed adjacency words, the edge table, and connected components (hook to
+// the smaller root + pointer jumping, so each root is its component's
+// minimum vertex and components rank by minimum vertex).
+#include "gb_internal.cuh"
+#include "../../include/graphb.h"
+
+#include <algorithm>
+#include <vector>
+
+namespace gb {
+
+// ---------------------------------------------------------------------------
+// Exclusive scan of uint32 (wrapping), three kernels: tile reduce, scan of the
+// tile sums in one CTA, tile scan + offset.
+// ---------------------------------------------------------------------------
+constexpr int kScanThreads = 256;
+constexpr int kScanItems = 8;
+constexpr int kScanTile = kScanThreads * kScanItems;
+
+__device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        uint32_t y = __shfl_up_sync(0xFFFFFFFFu, v, d);
+        if (lane >= d) v += y;
+    }
+    return v;
+}
+
+// block-wide exclusive scan of one value per thread; returns the block total
+__device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t &excl) {
+    __shared__ uint32_t wsum[32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    uint32_t incl = warp_incl_scan(v);
+    if (lane == 31) wsum[wid] = incl;
+    __syncthreads();
+    if (wid == 0) {
+        uint32_t s = lane < (int)(blockDim.x >> 5) ? wsum[lane] : 0;
+        s = warp_incl_scan(s);
+        wsum[lane] = s;
+    }
+    __syncthreads();
+    uint32_t base = wid ? wsum[wid - 1] : 0;
+    uint32_t total = wsum[(blockDim.x >> 5) - 1];
+    excl = base + incl - v;
+    __syncthreads();
+    return total;
+}
+
+__global__ void k_scan_reduce(const uint32_t *__restrict__ in, int64_t count,
+                              uint32_t *__restrict__ part) {
+    int64_t base = (int64_t)blockIdx.x * kScanTile;
+    uint32_t s = 0;
+#pragma unroll
+    for (int i = 0; i < kScanItems; i++) {
+        int64_t k = base + (int64_t)threadIdx.x * kScanItems + i;
+        if (k < count) s += in[k];
+    }
+    uint32_t ex;
+    uint32_t tot = block_excl_scan(s, ex);
+    if (threadIdx.x == 0) part[blockIdx.x] = tot;
+}
+
+__global__ void k_scan_partials(uint32_t *part, int64_t nparts) {
+    __shared__ uint32_t carry;
+    if (threadIdx.x == 0) carry = 0;
+    __syncthreads();
+    for (int64_t b = 0; b < nparts; b += blockDim.x) {
+        int64_t k = b + threadIdx.x;
+        uint32_t v = k < nparts ? part[k] : 0;
+        uint32_t ex;
+        uint32_t tot = block_excl_scan(v, ex);
+        if (k < nparts) part[k] = carry + ex;
+        __syncthreads();
+        if (threadIdx.x == 0) carry += tot;
+        __syncthreads();
+    }
+}
+
+__global__ void k_scan_down(const uint32_t *__restrict__ in, uint32_t *__restrict__ out,
+                            int64_t count, const uint32_t *__restrict__ part) {
+    int64_t base = (int64_t)blockIdx.x * kScanTile + (int64_t)threadIdx.x * kScanItems;
+    uint32_t v[kScanItems];
+    uint32_t s = 0;
+#pragma unroll
+    for (int i = 0; i < kScanItems; i++) {
+        v[i] = (base + i < count) ? in[base + i] : 0;
+        s += v[i];
+    }
+    uint32_t ex;
+    block_excl_scan(s, ex);
+    uint32_t run = part[blockIdx.x] + ex;
+#pragma unroll
+    for (int i = 0; i < kScanItems; i++) {
+        if (base + i < count) out[base + i] = run;
+        run += v[i];
+    }
+}
+
+size_t scan_tmp_elems(int64_t count) { return (size_t)((count + kScanTile - 1) / kScanTile) + 1; }
+
+int exclusive_scan_u32(const uint32_t *in, uint32_t *out, int64_t count, uint32_t *tmp,
+                       size_t tmp_elems, cudaStream_t st, int64_t *launches) {
+    if (count <= 0) return GB_OK;
+    int64_t nb = (count + kScanTile - 1) / kScanTile;
+    if ((size_t)nb > tmp_elems) { set_error("scan workspace too small"); return GB_ENOMEM; }
+    k_scan_reduce<<<(unsigned)nb, kScanThreads, 0, st>>>(in, count, tmp);
+    k_scan_partials<<<1, 1024, 0, st>>>(tmp, nb);
+    k_scan_down<<<(unsigned)nb, kScanThreads, 0, st>>>(in, out, count, tmp);
+    *launches += 3;
+    GB_CUDA_TRY(cudaGetLastError());
+    return GB_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Validation + edge ids
+// ---------------------------------------------------------------------------
+enum : uint32_t {
+    kErrRowPtr = 1u << 0, kErrColRange = 1u << 1, kErrSelfLoop = 1u << 2,
+    kErrUnsorted = 1u << 3, kErrSign = 1u << 4, kErrMirror = 1u << 5,
+    kErrMirrorSign = 1u << 6,
+};
+
+__global__ void k_rowptr(const int64_t *__restrict__ rp64, int64_t n, int64_t slots,
+                         uint32_t *__restrict__ rp, uint32_t *err) {
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u <= n;
+         u += (int64_t)gridDim.x * blockDim.x) {
+        int64_t a = rp64[u];
+        bool bad = a < 0 || a > slots || (u < n && rp64[u + 1] < a);
+        if (u == 0 && a != 0) bad = true;
+        if (u == n && a != slots) bad = true;
+        if (bad) atomicOr(err, kErrRowPtr);
+        rp[u] = (uint32_t)(bad ? 0 : a);
+    }
+}
+
+// row containing slot j: largest u with rp[u] <= j (rows may be empty)
+__device__ __forceinline__ uint32_t row_of_slot(const uint32_t *__restrict__ rp, int64_t n,
+                                                uint32_t j) {
+    uint32_t lo = 0, hi = (uint32_t)n;  // rp[lo] <= j < rp[hi]
+    while (hi - lo > 1) {
+        uint32_t mid = lo + ((hi - lo) >> 1);
+        if (__ldg(rp + mid) <= j) lo = mid; else hi = mid;
+    }
+    return lo;
+}
+
+// position of value x in the sorted row u, or kNone
+__device__ __forceinline__ uint32_t find_in_row(const uint32_t *__restrict__ rp,
+                                                const int32_t *__restrict__ col, uint32_t u,
+                                                int32_t x) {
+    uint32_t lo = __ldg(rp + u), hi = __ldg(rp + u + 1);
+    while (lo < hi) {
+        uint32_t mid = lo + ((hi - lo) >> 1);
+        int32_t c = __ldg(col + mid);
+        if (c == x) return mid;
+        if (c < x) lo = mid + 1; else hi = mid;
+    }
+    return kNone;
+}
+
+// first slot of row u whose column exceeds u (the upper part of the row)
+__global__ void k_upper(const uint32_t *__restrict__ rp, const int32_t *__restrict__ col,
+                        int64_t n, uint32_t *__restrict__ uptr, uint32_t *__restrict__ upc) {
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n;
+         u += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t lo = rp[u], hi = rp[u + 1], end = hi;
+        while (lo < hi) {
+            uint32_t mid = lo + ((hi - lo) >> 1);
+            if (col[mid] <= (int32_t)u) lo = mid + 1; else hi = mid;
+        }
+        uptr[u] = lo;
+        upc[u] = end - lo;
+    }
+}
+
+__global__ void k_slots(const uint32_t *__restrict__ rp, const int32_t *__restrict__ col,
+                        const int8_t *__restrict__ sign, int64_t n, uint64_t slots,
+                        const uint32_t *__restrict__ uptr, const uint32_t *__restrict__ ebase,
+                        uint32_t *__restrict__ adj, uint32_t *__restrict__ adj_eid,
+                        uint2 *__restrict__ edges, uint32_t *err) {
+    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < slots;
+         j += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t u = row_of_slot(rp, n, (uint32_t)j);
+        int32_t v = col[j];
+        int8_t s = sign[j];
+        uint32_t e = 0;
+        uint32_t bad = 0;
+        if (v < 0 || v >= n) bad |= kErrColRange;
+        if (v == (int32_t)u) bad |= kErrSelfLoop;
+        if (j > rp[u] && col[j - 1] >= v) bad |= kErrUnsorted;
+        if (s != 1 && s != -1) bad |= kErrSign;
+        if (!(bad & kErrColRange)) {
+            uint32_t mj = find_in_row(rp, col, (uint32_t)v, (int32_t)u);
+            if (mj == kNone) bad |= kErrMirror;
+            else {
+                if (sign[mj] != s) bad |= kErrMirrorSign;
+                if (v > (int32_t)u) e = ebase[u] + ((uint32_t)j - uptr[u]);
+                else e = ebase[v] + (mj - uptr[v]);
+            }
+        }
+        if (bad) { atomicOr(err, bad); continue; }
+        uint32_t negb = s < 0 ? kNegBit : 0u;
+        adj[j] = (uint32_t)v | negb;
+        adj_eid[j] = e;
+        if (v > (int32_t)u) edges[e] = make_uint2(u, (uint32_t)v | negb);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// Connected components: hook the larger root under the smaller one, with
+// pointer jumping (each final root = minimum vertex of its component).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ int32_t cc_find(int32_t *lab, int32_t x) {
+    while (true) {
+        int32_t p = ((volatile int32_t *)lab)[x];
+        if (p == x) return x;
+        int32_t gp = ((volatile int32_t *)lab)[p];
+        if (p != gp) ((volatile int32_t *)lab)[x] = gp;
+        x = p;
+    }
+}
+
+__global__ void k_cc_init(int32_t *lab, int64_t n) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+         v += (int64_t)gridDim.x * blockDim.x)
+        lab[v] = (int32_t)v;
+}
+
+__global__ void k_cc_hook(const uint2 *__restrict__ edges, int64_t m, int32_t *lab) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        uint2 ed = edges[e];
+        int32_t a = cc_find(lab, (int32_t)ed.x), b = cc_find(lab, (int32_t)(ed.y & kIdMask));
+        while (a != b) {
+            if (a < b) { int32_t t = a; a = b; b = t; }
+            int32_t old = atomicCAS(lab + a, a, b);
+            if (old == a) break;
+            a = cc_find(lab, old);
+            b = cc_find(lab, b);
+        }
+    }
+}
+
+// final roots go to a separate array: other threads' pointer jumping may still
+// write lab[] while this kernel runs
+__global__ void k_cc_finish(int32_t *lab, int64_t n, uint32_t *is_root, uint32_t *root) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        int32_t r = cc_find(lab, (int32_t)v);
+        root[v] = (uint32_t)r;
+        is_root[v] = (r == (int32_t)v) ? 1u : 0u;
+    }
+}
+
+__global__ void k_cc_rank(const uint32_t *__restrict__ root, const uint32_t *__restrict__ rank,
+                          int64_t n, int32_t *__restrict__ comp) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+         v += (int64_t)gridDim.x * blockDim.x)
+        comp[v] = (int32_t)rank[root[v]];
+}
+
+static unsigned grid_for(int64_t work, int threads, int sms) {
+    int64_t b = (work + threads - 1) / threads;
+    int64_t cap = (int64_t)sms * 16;
+    if (b > cap) b = cap;
+    if (b < 1) b = 1;
+    return (unsigned)b;
+}
+
+static const char *err_text(uint32_t f) {
+    if (f & kErrRowPtr) return "row_ptr must start at 0, be non-decreasing and end at 2m";
+    if (f & kErrColRange) return "column index out of range";
+    if (f & kErrSelfLoop) return "self loop";
+    if (f & kErrUnsorted) return "row not strictly increasing (unsorted or duplicate entry)";
+    if (f & kErrSign) return "sign must be +1 or -1";
+    if (f & kErrMirror) return "missing mirror entry (graph not symmetric)";
+    if (f & kErrMirrorSign) return "mirror entry has a different sign";
+    return "invalid graph";
+}
+
+int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32_t *h_col,
+           const int8_t *h_sign, cudaStream_t st, int64_t *launches) {
+    const uint64_t slots = 2ull * (uint64_t)m;
+    const int sms = g.num_sms;
+    int64_t *d_rp64 = nullptr;
+    int32_t *d_col = nullptr, *lab = nullptr;
+    int8_t *d_sign = nullptr;
+    uint32_t *d_err = nullptr, *uptr = nullptr, *upc = nullptr, *ebase = nullptr,
+             *tmp = nullptr, *flag = nullptr, *rank = nullptr;
+    int rc = GB_OK;
+    uint32_t h_err = 0;
+    size_t ntmp = scan_tmp_elems(std::max<int64_t>(n, 1));
+    auto fail = [&](int code) { rc = code; };
+#define ING_TRY(expr)                                                          \
+    do {                                                                       \
+        cudaError_t _e = (expr);                                               \
+        if (_e != cudaSuccess) {                                               \
+            set_error(std::string(#expr) + ": " + cudaGetErrorString(_e));     \
+            fail(_e == cudaErrorMemoryAllocation ? GB_ENOMEM : GB_ECUDA);      \
+            goto done;                                                         \
+        }                                                                      \
+    } while (0)
+    ING_TRY(cudaMalloc(&d_rp64, sizeof(int64_t) * (n + 1)));
+    ING_TRY(cudaMalloc(&d_col, sizeof(int32_t) * std::max<uint64_t>(slots, 1)));
+    ING_TRY(cudaMalloc(&d_sign, std::max<uint64_t>(slots, 1)));
+    ING_TRY(cudaMalloc(&d_err, sizeof(uint32_t)));
+    ING_TRY(cudaMalloc(&g.row_ptr, sizeof(uint32_t) * (n + 1)));
+    ING_TRY(cudaMalloc(&g.adj, sizeof(uint32_t) * std::max<uint64_t>(slots, 1)));
+    ING_TRY(cudaMalloc(&g.adj_eid, sizeof(uint32_t) * std::max<uint64_t>(slots, 1)));
+    ING_TRY(cudaMalloc(&g.edges, sizeof(uint2) * std::max<int64_t>(m, 1)));
+    ING_TRY(cudaMalloc(&g.comp, sizeof(int32_t) * n));
+    ING_TRY(cudaMalloc(&g.cverts, sizeof(int32_t) * n));
+    ING_TRY(cudaMalloc(&uptr, sizeof(uint32_t) * n));
+    ING_TRY(cudaMalloc(&upc, sizeof(uint32_t) * n));
+    ING_TRY(cudaMalloc(&ebase, sizeof(uint32_t) * n));
+    ING_TRY(cudaMalloc(&tmp, sizeof(uint32_t) * ntmp));
+    ING_TRY(cudaMalloc(&lab, sizeof(int32_t) * n));
+    ING_TRY(cudaMalloc(&flag, sizeof(uint32_t) * n));
+    ING_TRY(cudaMalloc(&rank, sizeof(uint32_t) * n));
+    ING_TRY(cudaMemcpyAsync(d_rp64, h_row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, st));
+    if (slots) {
+        ING_TRY(cudaMemcpyAsync(d_col, h_col, sizeof(int32_t) * slots, cudaMemcpyHostToDevice, st));
+        ING_TRY(cudaMemcpyAsync(d_sign, h_sign, slots, cudaMemcpyHostToDevice, st));
+    }
+    ING_TRY(cudaMemsetAsync(d_err, 0, sizeof(uint32_t), st));
+    k_rowptr<<<grid_for(n + 1, 256, sms), 256, 0, st>>>(d_rp64, n, (int64_t)slots, g.row_ptr, d_err);
+    ++*launches;
+    ING_TRY(cudaMemcpyAsync(&h_err, d_err, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+    ING_TRY(cudaStreamSynchronize(st));
+    if (h_err) { set_error(err_text(h_err)); fail(GB_EINVAL); goto done; }
+    k_upper<<<grid_for(n, 256, sms), 256, 0, st>>>(g.row_ptr, d_col, n, uptr, upc);
+    ++*launches;
+    rc = exclusive_scan_u32(upc, ebase, n, tmp, ntmp, st, launches);
+    if (rc) goto done;
+    if (slots) {
+        k_slots<<<grid_for((int64_t)slots, 256, sms), 256, 0, st>>>(
+            g.row_ptr, d_col, d_sign, n, slots, uptr, ebase, g.adj, g.adj_eid, g.edges, d_err);
+        ++*launches;
+    }
+    ING_TRY(cudaMemcpyAsync(&h_err, d_err, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+    ING_TRY(cudaStreamSynchronize(st));
+    if (h_err) { set_error(err_text(h_err)); fail(GB_EINVAL); goto done; }
+    // connected components
+    k_cc_init<<<grid_for(n, 256, sms), 256, 0, st>>>(lab, n);
+    ++*launches;
+    if (m) {
+        k_cc_hook<<<grid_for(m, 256, sms), 256, 0, st>>>(g.edges, m, lab);
+        ++*launches;
+    }
+    k_cc_finish<<<grid_for(n, 256, sms), 256, 0, st>>>(lab, n, flag, ebase);
+    ++*launches;
+    rc = exclusive_scan_u32(flag, rank, n, tmp, ntmp, st, launches);
+    if (rc) goto done;
+    k_cc_rank<<<grid_for(n, 256, sms), 256, 0, st>>>(ebase, rank, n, g.comp);
+    ++*launches;
+    {
+        // component offsets and ascending member lists: a counting sort of the
+        // n labels on the host (one-off, O(n))
+        std::vector<int32_t> hc(n);
+        ING_TRY(cudaMemcpyAsync(hc.data(), g.comp, sizeof(int32_t) * n, cudaMemcpyDeviceToHost, st));
+        ING_TRY(cudaStreamSynchronize(st));
+        int64_t nc = 0;
+        for (int64_t v = 0; v < n; v++) nc = std::max<int64_t>(nc, (int64_t)hc[v] + 1);
+        std::vector<int32_t> coff(nc + 1, 0), fill;
+        for (int64_t v = 0; v < n; v++) coff[hc[v] + 1]++;
+        int32_t big = 0;
+        for (int64_t c = 0; c < nc; c++) if (coff[c + 1] > coff[big + 1]) big = (int32_t)c;
+        for (int64_t c = 0; c < nc; c++) coff[c + 1] += coff[c];
+        fill.assign(coff.begin(), coff.end());
+        std::vector<int32_t> cv(n);
+        for (int64_t v = 0; v < n; v++) cv[fill[hc[v]]++] = (int32_t)v;
+        g.ncomp = nc;
+        g.cbig = big;
+        ING_TRY(cudaMalloc(&g.coff, sizeof(int32_t) * (nc + 1)));
+        ING_TRY(cudaMemcpyAsync(g.coff, coff.data(), sizeof(int32_t) * (nc + 1), cudaMemcpyHostToDevice, st));
+        ING_TRY(cudaMemcpyAsync(g.cverts, cv.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice, st));
+        ING_TRY(cudaStreamSynchronize(st));
+    }
+    g.n = n;
+    g.m = m;
+    g.slots = slots;
+done:
+#undef ING_TRY
+    cudaFree(d_rp64); cudaFree(d_col); cudaFree(d_sign); cudaFree(d_err);
+    cudaFree(uptr); cudaFree(upc); cudaFree(ebase); cudaFree(tmp); cudaFree(lab);
+    cudaFree(flag); cudaFree(rank);
+    return rc;
+}
+
+}  // namespace gb

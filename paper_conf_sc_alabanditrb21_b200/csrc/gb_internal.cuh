@@ -1,0 +1,148 @@
+// gb_internal.cuh -- shared definitions of the graphB+ B200 library (not part
+// of the C ABI).  Layout of the device state is documented in DESIGN.md
+// "Data layout in HBM".
+#pragma once
+#include <cuda_runtime.h>
+#include <cooperative_groups.h>
+#include <stdint.h>
+#include <string>
+
+namespace gb {
+
+constexpr uint32_t kNegBit = 0x80000000u;   // sign bit packed next to a 31-bit id (L238)
+constexpr uint32_t kIdMask = 0x7FFFFFFFu;
+constexpr int32_t kInf = 0x7F7F7F7F;         // "unvisited" BFS distance (memset 0x7F)
+constexpr uint32_t kNone = 0xFFFFFFFFu;
+constexpr int kMaxBatch = 64;                // trees per batch (smem tables)
+constexpr int kBlock = 256;                  // threads per CTA of the cooperative kernels
+
+// ---------------------------------------------------------------------------
+// Counter-based hash: SplitMix64 finaliser and its inverse (R4).
+// tkey(seed,t) = mix(seed + G*(t+1)); rkey = mix(tkey ^ (K*(C+1)));
+// ekey = mix(tkey + G*(e+1)).  mix is a bijection on 64-bit words, so an edge
+// key decodes back to the edge id: e = (unmix(key) - tkey) * G^-1 - 1.
+// ---------------------------------------------------------------------------
+constexpr uint64_t kGolden = 0x9E3779B97F4A7C15ull;
+constexpr uint64_t kGoldenInv = 0xF1DE83E19937733Dull;
+constexpr uint64_t kMul1 = 0xBF58476D1CE4E5B9ull, kMul1Inv = 0x96DE1B173F119089ull;
+constexpr uint64_t kMul2 = 0x94D049BB133111EBull, kMul2Inv = 0x319642B2D24D8EC3ull;
+constexpr uint64_t kRootMul = 0xD1B54A32D192ED03ull;
+
+__host__ __device__ __forceinline__ uint64_t mix64(uint64_t z) {
+    z ^= z >> 30; z *= kMul1;
+    z ^= z >> 27; z *= kMul2;
+    z ^= z >> 31;
+    return z;
+}
+__host__ __device__ __forceinline__ uint64_t unmix64(uint64_t z) {
+    z ^= (z >> 31) ^ (z >> 62); z *= kMul2Inv;
+    z ^= (z >> 27) ^ (z >> 54); z *= kMul1Inv;
+    z ^= (z >> 30) ^ (z >> 60);
+    return z;
+}
+__host__ __device__ __forceinline__ uint64_t tree_key(uint64_t seed, int64_t t) {
+    return mix64(seed + kGolden * (uint64_t)(t + 1));
+}
+__host__ __device__ __forceinline__ uint64_t root_key(uint64_t tkey, int64_t comp) {
+    return mix64(tkey ^ (kRootMul * (uint64_t)(comp + 1)));
+}
+__host__ __device__ __forceinline__ uint64_t edge_key(uint64_t tkey, uint32_t e) {
+    return mix64(tkey + kGolden * ((uint64_t)e + 1));
+}
+__host__ __device__ __forceinline__ uint32_t edge_of_key(uint64_t tkey, uint64_t key) {
+    return (uint32_t)((unmix64(key) - tkey) * kGoldenInv - 1);
+}
+
+// ---------------------------------------------------------------------------
+// Loaded graph (device arrays; immutable after gb_load_csr).  L236: a single
+// compact CSR; L238: sign bits packed next to 31-bit vertex ids.
+// ---------------------------------------------------------------------------
+struct Graph {
+    int64_t n = 0, m = 0, ncomp = 0;
+    uint64_t slots = 0;                 // 2m
+    uint32_t *row_ptr = nullptr;        // [n+1]
+    uint32_t *adj = nullptr;            // [2m] col | neg<<31
+    uint32_t *adj_eid = nullptr;        // [2m] eid of the slot
+    uint2 *edges = nullptr;             // [m] {u, v | neg<<31}, u < v, index = eid
+    int32_t *comp = nullptr;            // [n] component rank (by minimum vertex)
+    int32_t *coff = nullptr;            // [ncomp+1] component offsets (pre of the root)
+    int32_t *cverts = nullptr;          // [n] vertices grouped by component, ascending
+    int32_t cbig = 0;                   // largest component
+    int dev = 0;
+    int num_sms = 148;
+};
+
+// Per-batch workspace for B trees (arrays are [B][n] unless noted).
+struct Workspace {
+    int B = 0;                 // capacity in trees
+    int64_t n = 0;
+    int32_t *dist = nullptr;   // BFS level (kInf = unvisited)
+    uint64_t *pkey = nullptr;  // running min edge key of the parent candidates
+    unsigned long long *sz = nullptr; // packed (#children << 32 | subtree size) (Alg. 4 v_cnt)
+    uint32_t *qv = nullptr;    // level lists (vertices in BFS level order)
+    uint32_t *qs = nullptr;    // slot prefix of each queued vertex within its level
+    uint64_t *lvl = nullptr;   // [B][n+2] packed (vertex count << 32 | slot count) per level
+    uint32_t *vbase = nullptr; // [B][n+2] start of each level in qv
+    uint32_t *pinfo = nullptr; // parent id | neg(parent edge)<<31 (kNone at roots)
+    uint32_t *peid = nullptr;  // eid of the parent edge (kNone at roots)
+    uint32_t *off = nullptr;   // offset of a child's pre inside its parent's range
+    uint32_t *pp = nullptr;    // pre | pi<<31  (pi = root-path parity)
+    uint2 *rec = nullptr;      // [B][n] pre-indexed {up pre | neg<<31, size}
+    uint32_t *fbits = nullptr; // [B][ceil(m/32)] flip bitmask
+    uint32_t *s1 = nullptr;    // [B][ncomp] #vertices with pi = 1 per component
+    uint64_t *tkey = nullptr;  // [B]
+    int32_t *depth = nullptr;  // [B]
+    unsigned long long *tstat = nullptr; // [B][2] {sum cycle length, cycles}
+    int32_t *maxd = nullptr;   // [1] max depth over the batch
+    // descent variant (walk = 1)
+    uint32_t *cidx = nullptr;  // [B][n] sibling index of each child
+    uint32_t *cstart = nullptr;// [B][n] start of the child list (global position)
+    uint32_t *clist = nullptr; // [B*n] children pre IDs, grouped by parent, ascending
+    uint2 *crec = nullptr;     // [B][n] pre-indexed {cstart, #children}
+    uint32_t *scan_tmp = nullptr;
+    size_t scan_tmp_elems = 0;
+};
+
+struct BatchArgs {
+    int B;                 // trees in this batch
+    int64_t n, m;
+    int64_t ncomp;
+    uint64_t slots;
+};
+
+// ---------------------------------------------------------------------------
+// Error handling
+// ---------------------------------------------------------------------------
+void set_error(const std::string &msg);
+
+#define GB_CUDA_TRY(expr)                                                       \
+    do {                                                                         \
+        cudaError_t _e = (expr);                                                 \
+        if (_e != cudaSuccess) {                                                 \
+            ::gb::set_error(std::string(#expr) + ": " + cudaGetErrorString(_e)); \
+            return GB_ECUDA;                                                     \
+        }                                                                        \
+    } while (0)
+
+// ---------------------------------------------------------------------------
+// Launch helpers implemented in the .cu files
+// ---------------------------------------------------------------------------
+int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr,
+           const int32_t *h_col, const int8_t *h_sign, cudaStream_t st,
+           int64_t *launches);
+
+int run_batch_tree(const Graph &g, Workspace &ws, int B, const uint64_t *tkeys_host,
+                   const int32_t *given_parent, cudaStream_t st, int64_t *launches,
+                   cudaEvent_t *ev, bool walk_descent);
+
+int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool descent,
+                     cudaStream_t st, int64_t *launches);
+
+int run_batch_accumulate(const Graph &g, Workspace &ws, int B, int32_t *d_cnt,
+                         int32_t *d_agree, cudaStream_t st, int64_t *launches);
+
+int exclusive_scan_u32(const uint32_t *in, uint32_t *out, int64_t count, uint32_t *tmp,
+                       size_t tmp_elems, cudaStream_t st, int64_t *launches);
+size_t scan_tmp_elems(int64_t count);
+
+}  // namespace gb

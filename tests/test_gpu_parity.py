@@ -1,0 +1,302 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the
+same seeded inputs.  Everything here is integer work, so the bar is
+bit-exact: edge flip counts, vertex agree counts, per-tree sums of cycle
+lengths and cycle counts, and every stage of single trees (parent, dist,
+size, flips).  Pre-order IDs are not unique (the sibling order is free,
+reading R5), so they are checked for validity instead."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import graphgen
+import oracle
+from paper_conf_sc_alabanditrb21_b200 import graphb
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(autouse=True)
+def _reset_options():
+    yield
+    for k in ("batch", "cycle_group", "walk", "timing"):
+        graphb.set_option(k, 0)
+
+
+def check_cloud(g, T, seed, **opts):
+    for k, v in opts.items():
+        graphb.set_option(k, v)
+    graphb.load_graph(g)
+    cnt, agree = graphb.balance_host(T, seed)
+    st = graphb.stats()
+    ids, per = graphb.tree_stats()
+    og = oracle.Graph.from_csr(g)
+    ocnt, oagree, ostats = og.balance(T, seed, with_stats=True)
+    assert np.array_equal(cnt, ocnt), "edge flip counts"
+    assert np.array_equal(agree, oagree), "vertex agree"
+    assert list(ids) == list(range(T))
+    assert np.array_equal(per[:, 0], ostats[:, 0]), "per-tree sum of cycle lengths"
+    assert np.array_equal(per[:, 1], ostats[:, 1]), "per-tree cycles"
+    assert np.array_equal(per[:, 2], ostats[:, 2]), "per-tree depth"
+    assert st["cycles"] == T * (g.m - g.n + og.ncomp)     # L112
+    return st
+
+
+def valid_preorder(parent, size, pre, comp_off_of_root):
+    n = len(parent)
+    assert sorted(pre.tolist()) == list(range(n))
+    roots = np.flatnonzero(parent < 0)
+    for r in roots:
+        assert pre[r] == comp_off_of_root[r]
+    ch = np.flatnonzero(parent >= 0)
+    p = parent[ch]
+    # child's range nested strictly inside the parent's (Alg. 4)
+    assert np.all(pre[ch] > pre[p])
+    assert np.all(pre[ch] + size[ch] <= pre[p] + size[p])
+    # siblings' ranges disjoint and tile the parent's range: sort children by pre
+    order = np.lexsort((pre[ch], p))
+    cs, ps = ch[order], p[order]
+    first = np.ones(len(cs), bool)
+    first[1:] = ps[1:] != ps[:-1]
+    exp = np.where(first, pre[ps] + 1, 0)
+    prev_end = np.r_[0, pre[cs][:-1] + size[cs][:-1]]
+    exp = np.where(first, exp, prev_end)
+    assert np.array_equal(pre[cs], exp)
+
+
+def check_tree_debug(g, seed, trees, walk=0):
+    graphb.set_option("walk", walk)
+    graphb.load_graph(g)
+    og = oracle.Graph.from_csr(g)
+    comp, coff, _ = og.components()
+    for t in trees:
+        d = graphb.tree_debug(t, seed)
+        parent, dist, _ = og.bfs_tree(seed, t)
+        flip, sk, nc, _ = og.balance_tree(parent)
+        opre, osize = og.preorder(parent)
+        assert np.array_equal(d["parent"], parent)
+        assert np.array_equal(d["dist"], dist)
+        assert np.array_equal(d["size"], osize)
+        assert np.array_equal(d["flip"], flip)
+        assert d["sum_cycle_len"] == sk and d["num_cycles"] == nc
+        valid_preorder(d["parent"], d["size"], d["pre"], coff[comp])
+
+
+# ---------------------------------------------------------------------------
+
+def test_c1_config_exact():
+    """BASELINE configs[0]: ER 10k / 50k, 30% negative, 1 tree, seed 1."""
+    g, T, _ = graphgen.config("c1")
+    st = check_cloud(g, T, 1)
+    assert st["trees"] == 1
+
+
+@pytest.mark.parametrize("walk", [0, 1])
+def test_tree_stages_match_oracle(walk):
+    g = graphgen.er(3000, 12000, 0.3, 4)
+    check_tree_debug(g, 5, range(6), walk=walk)
+
+
+@pytest.mark.parametrize("walk", [0, 1])
+def test_power_law_hubs_multi_batch(walk):
+    """Hubs (Chung-Lu) + several batches + cycle groups smaller than a batch."""
+    g = graphgen.chung_lu(20000, 90000, 2500, 0.75, 0.25, 3)
+    check_cloud(g, 37, 11, batch=16, cycle_group=5, walk=walk)
+
+
+def test_disconnected_forest_with_isolated_vertices():
+    g = graphgen.er(5000, 3000, 0.4, 2)     # many components, isolated vertices
+    check_cloud(g, 9, 3)
+    check_tree_debug(g, 3, range(3))
+
+
+@pytest.mark.parametrize("name", ["path", "star", "ring", "complete", "grid", "single", "pair",
+                                  "empty", "diamond", "bipartite_neg"])
+def test_degenerate_graphs(name):
+    g = {
+        "path": lambda: graphgen.path(100),
+        "star": lambda: graphgen.star(3000),
+        "ring": lambda: graphgen.ring(101, [0, 5, 7]),
+        "complete": lambda: graphgen.complete(40, lambda u, v: -1 if (u * v) % 3 == 1 else 1),
+        "grid": lambda: graphgen.grid2d(40, 50, 0.3, 1),
+        "single": lambda: graphgen.from_edge_list(1, []),
+        "pair": lambda: graphgen.from_edge_list(2, [(0, 1, -1)]),
+        "empty": lambda: graphgen.from_edge_list(7, []),
+        "diamond": graphgen.diamond,
+        "bipartite_neg": lambda: graphgen.bipartite_chung_lu(500, 300, 2000, 50, 80, 0.5, 0.6, 1.0, 1),
+    }[name]()
+    check_cloud(g, 12, 7)
+
+
+def test_deep_path_many_levels():
+    """A long path: depth ~ n/2 levels in one cooperative kernel."""
+    g = graphgen.path(20000)
+    check_cloud(g, 3, 1)
+
+
+def test_balanced_inputs_closed_form():
+    gb, colour = graphgen.planted_signs(graphgen.largest_cc(graphgen.er(4001, 20000, 0.0, 9)), 2)
+    graphb.load_graph(gb)
+    T = 10
+    cnt, agree = graphb.balance_host(T, 5)
+    assert cnt.sum() == 0
+    ones = int(colour.sum())
+    big = 1 if ones > gb.n - ones else 0
+    exp = np.where(colour == big, 2 * T, 0)
+    assert np.array_equal(agree, exp)
+
+
+def test_given_trees_match_oracle():
+    """Alg. 3 on arbitrary (non-BFS) spanning trees."""
+    g = graphgen.er(2000, 7000, 0.35, 6)
+    graphb.load_graph(g)
+    og = oracle.Graph.from_csr(g)
+    rng = np.random.default_rng(0)
+    u, v, _ = og.edges()
+    for trial in range(4):
+        # random spanning forest via union-find over shuffled edges
+        par = np.arange(g.n)
+
+        def find(x):
+            while par[x] != x:
+                par[x] = par[par[x]]
+                x = par[x]
+            return x
+        adj = [[] for _ in range(g.n)]
+        for e in rng.permutation(g.m):
+            a, b = find(u[e]), find(v[e])
+            if a != b:
+                par[a] = b
+                adj[u[e]].append(v[e]); adj[v[e]].append(u[e])
+        parent = np.full(g.n, -2, np.int32)
+        for s in range(g.n):
+            if parent[s] != -2:
+                continue
+            parent[s] = -1
+            stack = [s]
+            while stack:
+                x = stack.pop()
+                for y in adj[x]:
+                    if parent[y] == -2:
+                        parent[y] = x
+                        stack.append(y)
+        flip, sk, nc = graphb.balance_given_tree(parent)
+        oflip, osk, onc, _ = og.balance_tree(parent)
+        assert np.array_equal(flip, oflip) and sk == osk and nc == onc
+    # invalid trees are rejected
+    bad = parent.copy()
+    bad[np.flatnonzero(bad >= 0)[0]] = -1          # two roots in one component
+    with pytest.raises(graphb.GraphBError):
+        graphb.balance_given_tree(bad)
+    bad = parent.copy()
+    x = int(np.flatnonzero(bad >= 0)[0])
+    nonadj = [w for w in range(g.n) if w != x and w not in set(g.col[g.row_ptr[x]:g.row_ptr[x + 1]])]
+    bad[x] = nonadj[0]                              # parent not adjacent
+    with pytest.raises(graphb.GraphBError):
+        graphb.balance_given_tree(bad)
+
+
+def test_invalid_csr_rejected():
+    g = graphgen.diamond()
+    cases = []
+    c = g.col.copy(); c[0] = c[1]; cases.append((g.row_ptr, c, g.sign))
+    s = g.sign.copy(); s[0] = -s[0]; cases.append((g.row_ptr, g.col, s))
+    s = g.sign.copy(); s[0] = 0; cases.append((g.row_ptr, g.col, s))
+    c = g.col.copy(); c[0] = 0; cases.append((g.row_ptr, c, g.sign))
+    c = g.col.copy(); c[0] = 77; cases.append((g.row_ptr, c, g.sign))
+    rp = g.row_ptr.copy(); rp[1], rp[2] = rp[2], rp[1]; cases.append((rp, g.col, g.sign))
+    for rp, c, s in cases:
+        with pytest.raises(graphb.GraphBError) as ei:
+            graphb.load_csr(rp, c, s)
+        assert ei.value.rc == graphb.GB_EINVAL
+
+
+def test_sharded_ranges_sum_to_full():
+    """L248: disjoint tree subsets add up (simulated sharding on one GPU)."""
+    import torch
+    g = graphgen.chung_lu(8000, 40000, 900, 0.75, 0.2, 5)
+    graphb.load_graph(g)
+    T = 24
+    full_c, full_a = graphb.balance_host(T, 3)
+    for W in (2, 3, 8):
+        cnt = torch.zeros(g.m, dtype=torch.int32, device="cuda")
+        agr = torch.zeros(g.n, dtype=torch.int32, device="cuda")
+        for r in range(W):
+            graphb.balance_range(r, T, W, 3, cnt, agr)
+        torch.cuda.synchronize()
+        assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), full_c)
+        assert np.array_equal(agr.cpu().numpy().astype(np.uint32), full_a)
+
+
+def test_deterministic_repeat():
+    g = graphgen.chung_lu(10000, 50000, 1500, 0.75, 0.3, 8)
+    graphb.load_graph(g)
+    a = graphb.balance_host(20, 9)
+    b = graphb.balance_host(20, 9)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+
+
+# ---------------------------------------------------------------------------
+# BASELINE config sizes (the launch configuration bench.py times)
+# ---------------------------------------------------------------------------
+
+def test_c2_slashdot_full_cloud():
+    g, T, _ = graphgen.config("c2")
+    check_cloud(g, T, 1)
+
+
+def test_c4_epinions_tree_subset():
+    """C4 at full size: a strided subset of the 1000 trees, bit-exact."""
+    import torch
+    g, T, _ = graphgen.config("c4")
+    graphb.load_graph(g)
+    cnt = torch.zeros(g.m, dtype=torch.int32, device="cuda")
+    agr = torch.zeros(g.n, dtype=torch.int32, device="cuda")
+    graphb.balance_range(3, T, 97, 1, cnt, agr)      # trees 3, 100, 197, ...
+    torch.cuda.synchronize()
+    oc, oa = oracle.Graph.from_csr(g).balance(T, 1, t_begin=3, stride=97)
+    assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), oc)
+    assert np.array_equal(agr.cpu().numpy().astype(np.uint32), oa)
+
+
+@pytest.mark.slow
+def test_c3_amazon_sampled_trees():
+    """C3 (10M / 22M) at full size in bench's batch configuration: per-tree
+    statistics of the whole batch against invariants, and two sampled trees
+    bit-exact against the oracle."""
+    g, T, _ = graphgen.config("c3")
+    graphb.load_graph(g)
+    cnt, agree = graphb.balance_host(8, 1)
+    ids, per = graphb.tree_stats()
+    og = oracle.Graph.from_csr(g)
+    c = og.ncomp
+    assert np.all(per[:, 1] == g.m - g.n + c)                  # L112
+    assert np.all(agree <= 16) and cnt.max() <= 8
+    for t in (0, 5):
+        parent, dist, _ = og.bfs_tree(1, t)
+        flip, sk, nc, md = og.balance_tree(parent)
+        assert per[t, 0] == sk and per[t, 2] == md
+        d = graphb.tree_debug(t, 1)
+        assert np.array_equal(d["parent"], parent)
+        assert np.array_equal(d["flip"], flip)
+
+
+@pytest.mark.parametrize("which", ["er", "forest", "c2"])
+def test_ingest_edge_ids_and_components(which):
+    """§8 a.1: edge table by eid (rank of (min,max)), eid of every slot, and
+    component ranks (by minimum vertex) equal the oracle's plain definitions."""
+    g = {"er": lambda: graphgen.er(3000, 9000, 0.3, 1),
+         "forest": lambda: graphgen.er(5000, 3000, 0.4, 2),
+         "c2": lambda: graphgen.config("c2")[0]}[which]()
+    graphb.load_graph(g)
+    eu, ev, en, se, comp = graphb.graph_debug()
+    og = oracle.Graph.from_csr(g)
+    ou, ov, on = og.edges()
+    oc, _, _ = og.components()
+    assert np.array_equal(eu, ou) and np.array_equal(ev, ov) and np.array_equal(en, on)
+    rows = np.repeat(np.arange(g.n), np.diff(g.row_ptr))
+    key = np.minimum(rows, g.col).astype(np.int64) * g.n + np.maximum(rows, g.col)
+    okey = ou.astype(np.int64) * g.n + ov
+    assert np.array_equal(se, np.searchsorted(okey, key))
+    assert np.array_equal(comp, oc)
+    assert graphb.graph_info()[2] == og.ncomp
