@@ -48,6 +48,8 @@ def lib():
         L.or_tkey.restype = u64; L.or_tkey.argtypes = [u64, i64]
         L.or_rkey.restype = u64; L.or_rkey.argtypes = [u64, i64, i64]
         L.or_ekey.restype = u64; L.or_ekey.argtypes = [u64, i64, i64]
+        L.or_pscore.restype = ctypes.c_uint32
+        L.or_pscore.argtypes = [u64, i64, ctypes.c_int32, ctypes.c_int32]
         L.or_build.restype = ctypes.c_int
         L.or_build.argtypes = [i64, i64, P, P, P, ctypes.POINTER(P)]
         L.or_free.restype = None; L.or_free.argtypes = [P]
@@ -90,6 +92,10 @@ def rkey(seed, t, c):
 
 def ekey(seed, t, e):
     return int(lib().or_ekey(seed, t, e))
+
+
+def pscore(seed, t, a, b):
+    return int(lib().or_pscore(seed, t, a, b))
 
 
 class OracleError(RuntimeError):

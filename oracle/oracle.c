@@ -75,6 +75,14 @@ uint64_t or_ekey(uint64_t seed, int64_t t, int64_t eid)
     return or_mix64(or_tkey(seed, t) + OR_GOLDEN * (uint64_t)(eid + 1));
 }
 
+/* Parent score of the edge {a,b} in tree t (reading R4): the high 32 bits of
+ * mix64(tkey + G * (min(a,b) * 2^32 + max(a,b))). */
+uint32_t or_pscore(uint64_t seed, int64_t t, int32_t a, int32_t b)
+{
+    uint64_t lo = (uint64_t)(a < b ? a : b), hi = (uint64_t)(a < b ? b : a);
+    return (uint32_t)(or_mix64(or_tkey(seed, t) + OR_GOLDEN * ((lo << 32) | hi)) >> 32);
+}
+
 /* ------------------------------------------------------------------------ */
 /* Graph ingest: validation (DESIGN.md "Boundary" error list), the undirected
  * edge list (m = #undirected edges, Table 1 L342 reading R2), edge
@@ -223,8 +231,9 @@ void or_components(const or_graph *g, int32_t *comp, int64_t *coff, int32_t *cve
 /* Tree sampling, Alg. 2 with M = BFS (L116-L123, L130; "random BFS trees"
  * L479).  Reading R4: the root of component C in tree t is
  * cverts_C[rkey(seed,t,C) mod |C|]; dist is the level-synchronous BFS
- * distance; parent[w] is the neighbour u with dist[u] = dist[w]-1 whose edge
- * has the smallest ekey(seed,t,eid(u,w)) (smaller u on an equal key).       */
+ * distance; parent[w] is the neighbour u with dist[u] = dist[w]-1 that
+ * minimises (pscore(seed,t,u,w), u) -- the score first, the smaller vertex
+ * id on an equal score.                                                     */
 /* ------------------------------------------------------------------------ */
 int or_bfs_tree(const or_graph *g, uint64_t seed, int64_t t,
                 int32_t *parent, int32_t *dist, int32_t *peid)
@@ -249,13 +258,13 @@ int or_bfs_tree(const or_graph *g, uint64_t seed, int64_t t,
         parent[w] = -1;
         if (peid) peid[w] = -1;
         if (dist[w] == 0) continue;
-        uint64_t best = 0;
+        uint32_t best = 0;
         int32_t bu = -1;
         int64_t be = -1;
         for (int64_t j = g->row_ptr[w]; j < g->row_ptr[w + 1]; j++) {
             int32_t u = g->col[j];
             if (dist[u] != dist[w] - 1) continue;
-            uint64_t k = or_ekey(seed, t, g->slot_eid[j]);
+            uint32_t k = or_pscore(seed, t, u, (int32_t)w);
             if (bu < 0 || k < best || (k == best && u < bu)) { best = k; bu = u; be = g->slot_eid[j]; }
         }
         parent[w] = bu;

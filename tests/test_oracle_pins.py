@@ -50,6 +50,23 @@ def test_splitmix64_kat():
     assert [oracle.tkey(0, t) for t in range(len(kat))] == kat
 
 
+def test_pscore_is_symmetric_and_spread():
+    """The parent score depends on the unordered edge only, and its 32-bit
+    values are spread (ties are rare; they fall back to the smaller id)."""
+    rng = np.random.default_rng(3)
+    vals = set()
+    for _ in range(3000):
+        a, b = (int(x) for x in rng.integers(0, 2**31 - 1, 2))
+        s1 = oracle.pscore(9, 4, a, b)
+        assert s1 == oracle.pscore(9, 4, b, a)
+        vals.add(s1)
+    assert len(vals) >= 2990
+    # the score is the high word of mix64 over the packed pair (pinned mix64)
+    a, b = 5, 77
+    z = (oracle.tkey(1, 0) + 0x9E3779B97F4A7C15 * ((a << 32) | b)) % 2**64
+    assert oracle.pscore(1, 0, a, b) == oracle.mix64(z) >> 32
+
+
 def test_mix64_is_a_bijection_sample():
     xs = np.random.default_rng(1).integers(0, 2**63, 20000, dtype=np.int64)
     ys = {oracle.mix64(int(x)) for x in xs}
@@ -112,12 +129,12 @@ def test_bfs_dist_and_minhash_parent(seed):
         # every edge spans at most one level (BFS-tree property)
         for u, v, _ in edges:
             assert abs(d[u] - d[v]) <= 1
-        # brute-force argmin of ekey over neighbours one level up
+        # brute-force argmin of (pscore, u) over neighbours one level up
         for w in range(g.n):
             if d[w] == 0:
                 continue
             cands = [int(u) for u in g.col[g.row_ptr[w]:g.row_ptr[w + 1]] if d[u] == d[w] - 1]
-            best = min(cands, key=lambda u: (oracle.ekey(seed, t, eid[(min(u, w), max(u, w))]), u))
+            best = min(cands, key=lambda u: (oracle.pscore(seed, t, u, w), u))
             assert parent[w] == best
             assert peid[w] == eid[(min(best, w), max(best, w))]
         # spanning forest: n - c edges, acyclic (union-find)
