@@ -52,9 +52,10 @@ static State S;
 constexpr int64_t kRecCap = 1 << 16;  // per-tree statistics kept for gb_tree_stats
 
 static void free_ws(Workspace &w) {
-    void *ptrs[] = {w.dist, w.pkey, w.sz, w.qv, w.qs, w.lvl, w.vbase, w.pinfo, w.peid,
-                    w.off, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth, w.tstat, w.maxd,
-                    w.cidx, w.cstart, w.clist, w.crec, w.scan_tmp};
+    void *ptrs[] = {w.visw, w.lvw, w.qv, w.qs, w.qr, w.pkeyq, w.lvl, w.vbase, w.size, w.sz64,
+                    w.parq, w.offq, w.szq, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth,
+                    w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
+                    w.scan_tmp};
     for (void *p : ptrs) if (p) cudaFree(p);
     w = Workspace();
 }
@@ -67,8 +68,8 @@ static void free_graph(Graph &g) {
 
 static size_t per_tree_bytes(const Graph &g, bool descent) {
     const size_t n = (size_t)g.n;
-    size_t b = 64 * n + 12 * 2 + 4 * (size_t)((g.m + 31) / 32) + 4 * (size_t)g.ncomp;
-    if (descent) b += 20 * n;
+    size_t b = 61 * n + 32 + 4 * (size_t)((g.m + 31) / 32) + 4 * (size_t)g.ncomp;
+    if (descent) b += 24 * n;
     return b;
 }
 
@@ -83,23 +84,24 @@ static size_t per_tree_bytes(const Graph &g, bool descent) {
     } while (0)
 
 static int ensure_workspace(int B, bool descent) {
-    if (S.ws.B >= B && (!descent || S.ws_descent)) return GB_OK;
+    if (S.ws.B >= B && descent == S.ws_descent) return GB_OK;
     B = std::max(B, S.ws.B);
-    descent = descent || S.ws_descent;
     free_ws(S.ws);
     Workspace &w = S.ws;
     const Graph &g = S.g;
     const int64_t n = g.n, Bn = (int64_t)B * n, words = (g.m + 31) / 32;
-    ALLOC(w.dist, Bn);
-    ALLOC(w.pkey, Bn);
-    ALLOC(w.sz, Bn);
+    const int64_t nw = (n + 31) / 32;
+    ALLOC(w.visw, (int64_t)B * nw);
+    ALLOC(w.lvw, (int64_t)B * 4 * nw);
     ALLOC(w.qv, Bn);
     ALLOC(w.qs, Bn);
+    ALLOC(w.qr, Bn);
+    ALLOC(w.pkeyq, Bn);
     ALLOC(w.lvl, (int64_t)B * (n + 2));
     ALLOC(w.vbase, (int64_t)B * (n + 2));
-    ALLOC(w.pinfo, Bn);
-    ALLOC(w.peid, Bn);
-    ALLOC(w.off, Bn);
+    ALLOC(w.parq, Bn);
+    ALLOC(w.offq, Bn);
+    ALLOC(w.szq, Bn);
     ALLOC(w.pp, Bn);
     ALLOC(w.rec, Bn);
     ALLOC(w.fbits, (int64_t)B * words);
@@ -107,14 +109,18 @@ static int ensure_workspace(int B, bool descent) {
     ALLOC(w.tkey, kMaxBatch);
     ALLOC(w.depth, kMaxBatch);
     ALLOC(w.tstat, 2 * kMaxBatch);
+    ALLOC(w.visited, kMaxBatch);
     ALLOC(w.maxd, 1);
     if (descent) {
-        ALLOC(w.cidx, Bn);
+        ALLOC(w.sz64, Bn);
+        ALLOC(w.cidxq, Bn);
         ALLOC(w.cstart, Bn);
         ALLOC(w.clist, Bn);
         ALLOC(w.crec, Bn);
         w.scan_tmp_elems = scan_tmp_elems(Bn);
         ALLOC(w.scan_tmp, (int64_t)w.scan_tmp_elems);
+    } else {
+        ALLOC(w.size, Bn);
     }
     w.B = B;
     w.n = n;
@@ -163,7 +169,7 @@ static int auto_batch(int64_t ntrees) {
     int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk == 1));
     int64_t b = std::min<int64_t>({ntrees, (int64_t)kMaxBatch, std::max<int64_t>(bm, 1)});
     // large graphs: a few trees per batch already fill the GPU
-    if (S.g.n >= (1 << 22)) b = std::min<int64_t>(b, 8);
+    if (S.g.n >= (1 << 22)) b = std::min<int64_t>(b, 2);
     return (int)std::max<int64_t>(b, 1);
 }
 
@@ -212,7 +218,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, nb, seed, t0, stride);
         ++T.launches;
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 2 * nb, st));
-        rc = run_batch_tree(S.g, S.ws, nb, nullptr, nullptr, st, &T.launches, ev, descent);
+        rc = run_batch_tree(S.g, S.ws, nb, nullptr, st, &T.launches, ev, descent);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
         rc = run_batch_cycles(S.g, S.ws, nb, G, descent, st, &T.launches);
@@ -263,18 +269,17 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
     k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, 1, seed, t, 1);
     ++T.launches;
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 2, st));
-    rc = run_batch_tree(S.g, S.ws, 1, nullptr, d_given, st, &T.launches, nullptr, S.opt.walk == 1);
+    rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk == 1);
     if (rc) return rc;
     if (d_given) {
         unsigned long long vis = 0;
-        GB_CUDA_TRY(cudaMemcpyAsync(&vis, S.ws.tstat, sizeof(vis), cudaMemcpyDeviceToHost, st));
+        GB_CUDA_TRY(cudaMemcpyAsync(&vis, S.ws.visited, sizeof(vis), cudaMemcpyDeviceToHost, st));
         GB_CUDA_TRY(cudaStreamSynchronize(st));
         if ((int64_t)vis != S.g.n) {
             set_error("parent is not a spanning forest of the loaded graph (some vertex is not "
                       "reachable from a root through parent edges)");
             return GB_EINVAL;
         }
-        GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 2, st));
     }
     rc = run_batch_cycles(S.g, S.ws, 1, 1, S.opt.walk == 1, st, &T.launches);
     if (rc) return rc;
@@ -447,20 +452,21 @@ int gb_tree_debug(int64_t t, uint64_t seed, int32_t *parent, int32_t *dist, int3
     int rc = run_single_tree(t, seed, nullptr);
     if (rc) return rc;
     const int64_t n = S.g.n;
-    std::vector<uint32_t> tmp(n);
-    if (parent) {
-        GB_CUDA_TRY(cudaMemcpy(tmp.data(), S.ws.pinfo, 4 * n, cudaMemcpyDeviceToHost));
-        for (int64_t v = 0; v < n; v++) parent[v] = tmp[v] == kNone ? -1 : (int32_t)(tmp[v] & kIdMask);
-    }
-    if (dist) GB_CUDA_TRY(cudaMemcpy(dist, S.ws.dist, 4 * n, cudaMemcpyDeviceToHost));
+    int32_t *d_tmp = nullptr;
+    GB_CUDA_TRY(cudaMalloc(&d_tmp, sizeof(int32_t) * 3 * n));
+    rc = debug_tree_views(S.g, S.ws, S.opt.walk == 1, d_tmp, d_tmp + n, d_tmp + 2 * n, S.stream);
+    if (rc) { cudaFree(d_tmp); return rc; }
+    std::vector<int32_t> h(3 * n);
+    cudaError_t ce = cudaMemcpy(h.data(), d_tmp, sizeof(int32_t) * 3 * n, cudaMemcpyDeviceToHost);
+    cudaFree(d_tmp);
+    GB_CUDA_TRY(ce);
+    if (parent) std::copy(h.begin(), h.begin() + n, parent);
+    if (dist) std::copy(h.begin() + n, h.begin() + 2 * n, dist);
+    if (size) std::copy(h.begin() + 2 * n, h.end(), size);
     if (pre) {
+        std::vector<uint32_t> tmp(n);
         GB_CUDA_TRY(cudaMemcpy(tmp.data(), S.ws.pp, 4 * n, cudaMemcpyDeviceToHost));
         for (int64_t v = 0; v < n; v++) pre[v] = (int32_t)(tmp[v] & kIdMask);
-    }
-    if (size) {
-        std::vector<unsigned long long> s64(n);
-        GB_CUDA_TRY(cudaMemcpy(s64.data(), S.ws.sz, 8 * n, cudaMemcpyDeviceToHost));
-        for (int64_t v = 0; v < n; v++) size[v] = (int32_t)(uint32_t)s64[v];
     }
     if (flip) { rc = copy_flips(flip); if (rc) return rc; }
     return copy_cycle_stats(sum_cycle_len, num_cycles);

@@ -73,32 +73,37 @@ struct Graph {
 };
 
 // Per-batch workspace for B trees (arrays are [B][n] unless noted).
+// "q" = queue order (BFS level lists), "v" = vertex order, "pre" = pre order.
 struct Workspace {
     int B = 0;                 // capacity in trees
     int64_t n = 0;
-    int32_t *dist = nullptr;   // BFS level (kInf = unvisited)
-    uint64_t *pkey = nullptr;  // running min edge key of the parent candidates
-    unsigned long long *sz = nullptr; // packed (#children << 32 | subtree size) (Alg. 4 v_cnt)
-    uint32_t *qv = nullptr;    // level lists (vertices in BFS level order)
-    uint32_t *qs = nullptr;    // slot prefix of each queued vertex within its level
+    uint32_t *visw = nullptr;  // [B][n/32] visited bitmap
+    uint32_t *lvw = nullptr;   // [B][4][n/32] level-membership bitmaps (ring of 4)
+    uint32_t *qv = nullptr;    // q: level lists (vertices in BFS level order)
+    uint32_t *qs = nullptr;    // q: slot prefix of each queued vertex within its level
+    uint32_t *qr = nullptr;    // q: CSR row start of each queued vertex
+    unsigned long long *pkeyq = nullptr; // q: parent key (score<<32 | parent<<1 | neg)
     uint64_t *lvl = nullptr;   // [B][n+2] packed (vertex count << 32 | slot count) per level
     uint32_t *vbase = nullptr; // [B][n+2] start of each level in qv
-    uint32_t *pinfo = nullptr; // parent id | neg(parent edge)<<31 (kNone at roots)
-    uint32_t *peid = nullptr;  // eid of the parent edge (kNone at roots)
-    uint32_t *off = nullptr;   // offset of a child's pre inside its parent's range
-    uint32_t *pp = nullptr;    // pre | pi<<31  (pi = root-path parity)
-    uint2 *rec = nullptr;      // [B][n] pre-indexed {up pre | neg<<31, size}
+    uint32_t *size = nullptr;  // v: subtree size (Alg. 4 v_cnt), walk 0
+    unsigned long long *sz64 = nullptr; // v: (#children << 32 | subtree size), walk 1
+    uint32_t *parq = nullptr;  // q: parent id | neg(parent edge)<<31
+    uint32_t *offq = nullptr;  // q: offset of the child's range inside its parent's
+    uint32_t *szq = nullptr;   // q: subtree size
+    uint32_t *pp = nullptr;    // v: pre | pi<<31  (pi = root-path parity)
+    uint2 *rec = nullptr;      // pre: {up pre | neg<<31, size}
     uint32_t *fbits = nullptr; // [B][ceil(m/32)] flip bitmask
     uint32_t *s1 = nullptr;    // [B][ncomp] #vertices with pi = 1 per component
-    uint64_t *tkey = nullptr;  // [B]
-    int32_t *depth = nullptr;  // [B]
-    unsigned long long *tstat = nullptr; // [B][2] {sum cycle length, cycles}
+    uint64_t *tkey = nullptr;  // [kMaxBatch]
+    int32_t *depth = nullptr;  // [kMaxBatch]
+    unsigned long long *tstat = nullptr;   // [kMaxBatch][2] {sum cycle length, cycles}
+    unsigned long long *visited = nullptr; // [kMaxBatch] vertices reached (given trees)
     int32_t *maxd = nullptr;   // [1] max depth over the batch
-    // descent variant (walk = 1)
-    uint32_t *cidx = nullptr;  // [B][n] sibling index of each child
-    uint32_t *cstart = nullptr;// [B][n] start of the child list (global position)
+    // walk 1 (Alg. 3 descent)
+    uint32_t *cidxq = nullptr; // q: sibling index of each child (pre order)
+    uint32_t *cstart = nullptr;// v: start of the child list (global position)
     uint32_t *clist = nullptr; // [B*n] children pre IDs, grouped by parent, ascending
-    uint2 *crec = nullptr;     // [B][n] pre-indexed {cstart, #children}
+    uint2 *crec = nullptr;     // pre: {cstart, #children}
     uint32_t *scan_tmp = nullptr;
     size_t scan_tmp_elems = 0;
 };
@@ -131,9 +136,11 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr,
            const int32_t *h_col, const int8_t *h_sign, cudaStream_t st,
            int64_t *launches);
 
-int run_batch_tree(const Graph &g, Workspace &ws, int B, const uint64_t *tkeys_host,
-                   const int32_t *given_parent, cudaStream_t st, int64_t *launches,
-                   cudaEvent_t *ev, bool walk_descent);
+int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
+                   cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent);
+
+int debug_tree_views(const Graph &g, Workspace &ws, bool descent, int32_t *d_parent,
+                     int32_t *d_dist, int32_t *d_size, cudaStream_t st);
 
 int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool descent,
                      cudaStream_t st, int64_t *launches);
