@@ -85,7 +85,7 @@ struct Workspace {
     unsigned long long *pkeyq = nullptr; // q: parent key (score<<32 | parent<<1 | neg)
     uint64_t *lvl = nullptr;   // [B][n+2] packed (vertex count << 32 | slot count) per level
     uint32_t *vbase = nullptr; // [B][n+2] start of each level in qv
-    uint32_t *size = nullptr;  // v: subtree size (Alg. 4 v_cnt), walk 0
+    uint32_t *size = nullptr;  // v: sum of the children's subtree sizes (Alg. 4 v_cnt - 1), walk 0
     unsigned long long *sz64 = nullptr; // v: (#children << 32 | subtree size), walk 1
     uint32_t *parq = nullptr;  // q: parent id | neg(parent edge)<<31
     uint32_t *offq = nullptr;  // q: offset of the child's range inside its parent's

@@ -103,7 +103,6 @@ __device__ __forceinline__ void place_root(const TreeParams &P, int b, int64_t C
     const size_t nb = (size_t)b * P.n;
     atomicOr(P.visw + (size_t)b * P.nw + (r >> 5), 1u << (r & 31));
     atomicOr(P.lvw + (size_t)b * 4 * P.nw + (r >> 5), 1u << (r & 31));  // level 0
-    if (P.sz64) P.sz64[nb + r] = 1; else P.size[nb + r] = 1;
     const uint32_t deg = P.row_ptr[r + 1] - P.row_ptr[r];
     const uint32_t pre = (uint32_t)P.coff[C];
     if (deg == 0) {
@@ -178,7 +177,6 @@ __device__ __forceinline__ void flush_discoveries(const TreeParams &P, int b, ui
             P.qs[nb + pos + i] = run + incl - e.y;
             P.qr[nb + pos + i] = e.z;
             P.pkeyq[nb + pos + i] = ~0ull;
-            if (P.sz64) P.sz64[nb + e.x] = 1; else P.size[nb + e.x] = 1;
         }
         run += __shfl_sync(0xFFFFFFFFu, incl, 31);
     }
@@ -243,9 +241,12 @@ __device__ __forceinline__ void expand_range(const TreeParams &P, int b, int L, 
                     atomicOr(visw + word, bit);
                 }
             } else {
-                if (!(__ldcg(visw + word) & bit)) {
+                // both words are independent L2 hits: issue them together
+                const uint32_t vw = __ldcg(visw + word);
+                const uint32_t pw = __ldcg(lv_prev + word);
+                if (!(vw & bit)) {
                     disc = !(atomicOr(visw + word, bit) & bit);
-                } else if (L > 0 && (__ldcg(lv_prev + word) & bit)) {
+                } else if (pw & bit) {
                     // a neighbour one level up is a parent candidate of w (a.3)
                     key = parent_key(tk, x, w, neg);
                 }
@@ -287,7 +288,6 @@ __device__ __forceinline__ void expand_range(const TreeParams &P, int b, int L, 
                     P.qs[nb + pos] = (uint32_t)old + (incl - deg);
                     P.qr[nb + pos] = rs;
                     P.pkeyq[nb + pos] = ((unsigned long long)w << 1) | neg;
-                    if (P.sz64) P.sz64[nb + x] = 1; else P.size[nb + x] = 1;
                 }
             } else {
                 const uint32_t k = __popc(dm);
@@ -310,7 +310,7 @@ __device__ __forceinline__ void expand_range(const TreeParams &P, int b, int L, 
     if (nbuf) flush_discoveries(P, b, vb + nv, lvl_next, wbuf, nbuf);
 }
 
-__global__ void __launch_bounds__(kBlock, 5) k_bfs(TreeParams P) {
+__global__ void __launch_bounds__(kBlock, 6) k_bfs(TreeParams P) {
     cg::grid_group grid = cg::this_grid();
     __shared__ LevelTable T;
     __shared__ uint64_t s_tkey[kMaxBatch];
@@ -480,18 +480,19 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
                 const uint32_t k = (uint32_t)__ldcg(P.pkeyq + qi);
                 p = k >> 1;
                 neg = k << 31;
-                sz = kDescent ? (uint32_t)__ldcg(P.sz64 + nb + w) : __ldcg(P.size + nb + w);
+                // counters hold the sum of the children's sizes: size = 1 + that
+                sz = 1 + (kDescent ? (uint32_t)__ldcg(P.sz64 + nb + w) : __ldcg(P.size + nb + w));
             }
             if (kDescent) {
                 const unsigned long long o =
                     aggregated_add<unsigned long long>(P.sz64 + nb + p, (1ull << 32) | sz, valid);
                 if (valid) {
-                    P.offq[qi] = (uint32_t)o;
+                    P.offq[qi] = 1 + (uint32_t)o;
                     P.cidxq[qi] = (uint32_t)(o >> 32);
                 }
             } else {
                 const uint32_t o = aggregated_add<uint32_t>(P.size + nb + p, sz, valid);
-                if (valid) P.offq[qi] = o;
+                if (valid) P.offq[qi] = 1 + o;
             }
             if (valid) {
                 P.parq[qi] = p | neg;
@@ -540,7 +541,7 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
                 up = pre;
                 neg = 0;
                 pi = 0;
-                szx = kDescent ? (uint32_t)__ldcg(P.sz64 + nb + x) : __ldcg(P.size + nb + x);
+                szx = 1 + (kDescent ? (uint32_t)__ldcg(P.sz64 + nb + x) : __ldcg(P.size + nb + x));
             } else {
                 const uint32_t pq = __ldcg(P.parq + qi);
                 p = pq & kIdMask;
@@ -589,7 +590,7 @@ __global__ void k_debug_tree(TreeParams P, int32_t *parent, int32_t *dist, int32
          v += (int64_t)gridDim.x * blockDim.x) {
         parent[v] = -1;
         dist[v] = 0;
-        size[v] = P.sz64 ? (int32_t)(uint32_t)P.sz64[v] : (int32_t)P.size[v];
+        size[v] = 1 + (P.sz64 ? (int32_t)(uint32_t)P.sz64[v] : (int32_t)P.size[v]);
     }
 }
 
@@ -666,6 +667,8 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
     GB_CUDA_TRY(cudaMemsetAsync(ws.visw, 0, sizeof(uint32_t) * (size_t)B * nw, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.lvw, 0, sizeof(uint32_t) * (size_t)B * 4 * nw, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.s1, 0, sizeof(uint32_t) * (size_t)B * g.ncomp, st));
+    if (descent) GB_CUDA_TRY(cudaMemsetAsync(ws.sz64, 0, sizeof(unsigned long long) * (size_t)B * g.n, st));
+    else GB_CUDA_TRY(cudaMemsetAsync(ws.size, 0, sizeof(uint32_t) * (size_t)B * g.n, st));
     k_batch_prep<<<1, kMaxBatch, 0, st>>>(P);
     ++*launches;
     if (given_parent) {
