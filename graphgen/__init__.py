@@ -30,7 +30,7 @@ import numpy as np
 
 __all__ = [
     "SignedCSR", "csr_from_edges", "er", "chung_lu", "bipartite_chung_lu",
-    "rmat", "largest_cc", "permute", "config", "CONFIGS",
+    "rmat", "rmat_gpu", "largest_cc", "permute", "config", "CONFIGS",
     "ring", "path", "star", "complete", "grid2d", "diamond", "planted_signs",
     "random_tiny", "from_edge_list",
 ]
@@ -304,6 +304,63 @@ def rmat(scale, edge_factor, p_neg, seed, abcd=(0.57, 0.19, 0.19, 0.05),
     return _finish(n, u, v, _signs(rng, len(u), p_neg), seed, name, lcc=False)
 
 
+def rmat_gpu(scale, edge_factor, p_neg, seed, abcd=(0.57, 0.19, 0.19, 0.05),
+             name="rmat", chunk=1 << 26, device="cuda"):
+    """Graph500 R-MAT generated with torch on a CUDA device (the same recipe as
+    ``rmat``; a different random stream, so a different -- equally seeded --
+    graph).  For scale 26 the numpy version needs many minutes of host time.
+    Returns a SignedCSR with host (numpy) arrays."""
+    import torch
+    gen = torch.Generator(device=device)
+    gen.manual_seed(int(seed) * 1000003 + 4)
+    n = 1 << scale
+    total = edge_factor * n
+    a, b, c, _ = abcd
+    keys = []
+    done = 0
+    while done < total:
+        k = min(chunk, total - done)
+        src = torch.zeros(k, dtype=torch.int64, device=device)
+        dst = torch.zeros(k, dtype=torch.int64, device=device)
+        for bit in range(scale):
+            r = torch.rand(k, generator=gen, device=device)
+            src |= (r >= a + b).to(torch.int64) << bit
+            dst |= (((r >= a) & (r < a + b)) | (r >= a + b + c)).to(torch.int64) << bit
+        lo = torch.minimum(src, dst)
+        hi = torch.maximum(src, dst)
+        keep = lo != hi
+        keys.append(torch.unique(lo[keep] * n + hi[keep]))
+        del src, dst, lo, hi, keep
+        done += k
+    key = torch.unique(torch.cat(keys))
+    del keys
+    m = key.numel()
+    neg = (torch.rand(m, generator=gen, device=device) < p_neg).to(torch.int64)
+    perm = torch.randperm(n, generator=gen, device=device)
+    u = perm[key // n]
+    v = perm[key % n]
+    del key
+    lo = torch.minimum(u, v)
+    hi = torch.maximum(u, v)
+    del u, v
+    both = torch.cat([(lo * n + hi) * 2 + neg, (hi * n + lo) * 2 + neg])
+    del lo, hi, neg
+    both, _ = torch.sort(both)
+    sg = torch.where((both & 1).bool(), -1, 1).to(torch.int8)
+    both >>= 1
+    srcv = both // n
+    col = (both - srcv * n).to(torch.int32)
+    del both
+    cnt = torch.bincount(srcv, minlength=n)
+    del srcv
+    row_ptr = torch.zeros(n + 1, dtype=torch.int64, device=device)
+    row_ptr[1:] = torch.cumsum(cnt, 0)
+    out = SignedCSR(n, m, row_ptr.cpu().numpy(), col.cpu().numpy(), sg.cpu().numpy(), name)
+    del row_ptr, col, sg, cnt
+    torch.cuda.empty_cache()
+    return out
+
+
 # --------------------------------------------------------------------------
 # Tiny / structured graphs for tests
 # --------------------------------------------------------------------------
@@ -398,8 +455,8 @@ CONFIGS = {
     "c4w": (lambda seed=1: chung_lu(7_539, 112_058, 1_079, 0.6, 0.22, seed,
                                     name="c4w_wikielec"), 1000,
             "wiki-Elec-shaped power law, LCC of 7,539 / 112,058 generated, 1000 trees"),
-    "c5": (lambda seed=1: rmat(26, 16, 0.5, seed, name="c5_rmat26"), 10,
-           "RMAT scale 26, edge factor 16 (~1B generated edges), random signs, 10 trees"),
+    "c5": (lambda seed=1: rmat_gpu(26, 16, 0.5, seed, name="c5_rmat26"), 10,
+           "RMAT scale 26, edge factor 16 (~1B generated edges, GPU-generated), random signs, 10 trees"),
 }
 
 

@@ -54,6 +54,40 @@ __host__ __device__ __forceinline__ uint32_t edge_of_key(uint64_t tkey, uint64_t
 }
 
 // ---------------------------------------------------------------------------
+// L2 eviction-priority hints (createpolicy + ld/st .L2::cache_hint): the
+// per-tree label arrays gathered at random are kept (evict_last) while the
+// edge table streams through (evict_first).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t l2_keep_policy() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t l2_stream_policy() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint2 ld_hint(const uint2 *ptr, uint64_t pol) {
+    uint2 r;
+    asm volatile("ld.global.nc.L2::cache_hint.v2.u32 {%0, %1}, [%2], %3;"
+                 : "=r"(r.x), "=r"(r.y) : "l"(ptr), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ uint32_t ld_hint(const uint32_t *ptr, uint64_t pol) {
+    uint32_t r;
+    asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(ptr), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ void st_hint(uint2 *ptr, uint2 v, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.v2.u32 [%0], {%1, %2}, %3;"
+                 :: "l"(ptr), "r"(v.x), "r"(v.y), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void st_hint(uint32_t *ptr, uint32_t v, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.u32 [%0], %1, %2;" :: "l"(ptr), "r"(v), "l"(pol) : "memory");
+}
+
+// ---------------------------------------------------------------------------
 // Loaded graph (device arrays; immutable after gb_load_csr).  L236: a single
 // compact CSR; L238: sign bits packed next to 31-bit vertex ids.
 // ---------------------------------------------------------------------------

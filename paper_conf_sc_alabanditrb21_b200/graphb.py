@@ -122,14 +122,18 @@ def graph_info():
     return n.value, m.value, c.value
 
 
-def graph_debug():
-    """Ingest results (a.1): edge table by eid, eid of every slot, components."""
+def graph_debug(edges=True, slot_eid=True, comp=True):
+    """Ingest results (a.1): edge table by eid, eid of every slot, components
+    (arrays not asked for come back as None)."""
     n, m, _ = graph_info()
-    eu = np.zeros(max(m, 1), np.int32); ev = np.zeros(max(m, 1), np.int32)
-    en = np.zeros(max(m, 1), np.int8); se = np.zeros(max(2 * m, 1), np.uint32)
-    comp = np.zeros(n, np.int32)
-    _check(lib().gb_graph_debug(_ptr(eu), _ptr(ev), _ptr(en), _ptr(se), _ptr(comp)))
-    return eu[:m], ev[:m], en[:m], se[:2 * m], comp
+    eu = np.zeros(max(m, 1), np.int32) if edges else None
+    ev = np.zeros(max(m, 1), np.int32) if edges else None
+    en = np.zeros(max(m, 1), np.int8) if edges else None
+    se = np.zeros(max(2 * m, 1), np.uint32) if slot_eid else None
+    cp = np.zeros(n, np.int32) if comp else None
+    _check(lib().gb_graph_debug(_ptr(eu), _ptr(ev), _ptr(en), _ptr(se), _ptr(cp)))
+    cut = lambda a, k: a[:k] if a is not None else None
+    return cut(eu, m), cut(ev, m), cut(en, m), cut(se, 2 * m), cp
 
 
 def set_option(key: str, value: int):

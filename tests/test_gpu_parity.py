@@ -300,3 +300,80 @@ def test_ingest_edge_ids_and_components(which):
     assert np.array_equal(se, np.searchsorted(okey, key))
     assert np.array_equal(comp, oc)
     assert graphb.graph_info()[2] == og.ncomp
+
+
+def _climb_checks(g, d, sample_edges, rng):
+    """Closed-form checks of sampled edges of one tree (any size): tree edges
+    never flip; a non-tree edge flips iff pi(u) ^ pi(v) ^ neg(e) with pi the
+    XOR of negative bits on the root path (L214); the cycle length is
+    d(u) + d(v) - 2 d(lca) + 1 (L230)."""
+    parent, dist, flip = d["parent"], d["dist"], d["flip"]
+    rows = np.searchsorted(g.row_ptr, sample_edges, side="right") - 1
+    u = rows.astype(np.int64)
+    v = g.col[sample_edges].astype(np.int64)
+    neg = (g.sign[sample_edges] < 0).astype(np.int64)
+    keep = u < v
+    u, v, neg, slots = u[keep], v[keep], neg[keep], sample_edges[keep]
+    # eid of each sampled slot (a.1 ingest, itself checked against the oracle
+    # on smaller graphs by test_ingest_edge_ids_and_components)
+    eid = graphb.graph_debug(edges=False, comp=False)[3][slots].astype(np.int64)
+
+    def neg_of_parent_edge(x):
+        p = parent[x]
+        out = np.zeros(len(x), np.int64)
+        ok = p >= 0
+        xs, ps = x[ok], p[ok].astype(np.int64)
+        # sign of edge (x, p): search p in row x
+        pos = np.array([g.row_ptr[a] + np.searchsorted(g.col[g.row_ptr[a]:g.row_ptr[a + 1]], b)
+                        for a, b in zip(xs, ps)], np.int64)
+        out[ok] = (g.sign[pos] < 0)
+        return out
+    tree = (parent[v] == u) | (parent[u] == v)
+    assert np.all(flip[eid[tree]] == 0)
+    a, b = u[~tree].copy(), v[~tree].copy()
+    ne = neg[~tree]
+    c = np.zeros(len(a), np.int64)
+    k = np.ones(len(a), np.int64)
+    da, db = dist[a].astype(np.int64), dist[b].astype(np.int64)
+    while True:
+        live = a != b
+        if not live.any():
+            break
+        mova = live & (da >= db)
+        movb = live & ~mova
+        c[mova] ^= neg_of_parent_edge(a[mova]); a[mova] = parent[a[mova]]; da[mova] -= 1
+        c[movb] ^= neg_of_parent_edge(b[movb]); b[movb] = parent[b[movb]]; db[movb] -= 1
+        k[live] += 1
+    assert np.array_equal(flip[eid[~tree]], (c ^ ne).astype(np.uint8))
+    return int((~tree).sum()), k
+
+
+@pytest.mark.slow
+def test_c5_rmat26_capacity_and_sampled_cycles():
+    """C5 (RMAT scale 26, ~1 B generated edges) on one B200: loads, balances
+    whole trees, per-tree cycle count m - n + c (L112), counters bounded, and
+    sampled edges of one tree against the closed forms."""
+    g, T, _ = graphgen.config("c5")
+    graphb.load_graph(g)
+    n, m, c = graphb.graph_info()
+    assert (n, m) == (g.n, g.m)
+    cnt, agree = graphb.balance_host(2, 1)
+    ids, per = graphb.tree_stats()
+    assert np.all(per[:, 1] == m - n + c)
+    assert cnt.max() <= 2 and agree.max() <= 4
+    d = graphb.tree_debug(0, 1)
+    assert per[0, 0] == d["sum_cycle_len"]
+    rng = np.random.default_rng(5)
+    deg = np.diff(g.row_ptr)
+    # the parent rule on sampled low-degree vertices (oracle's pscore)
+    cand_v = rng.integers(0, g.n, 4000)
+    for w in cand_v[(deg[cand_v] > 0) & (deg[cand_v] < 200)][:300]:
+        w = int(w)
+        if d["parent"][w] < 0:
+            continue
+        nb = g.col[g.row_ptr[w]:g.row_ptr[w + 1]]
+        cands = [int(x) for x in nb if d["dist"][x] == d["dist"][w] - 1]
+        best = min(cands, key=lambda x: (oracle.pscore(1, 0, x, w), x))
+        assert d["parent"][w] == best
+    nonc, _ = _climb_checks(g, d, rng.integers(0, len(g.col), 20000), rng)
+    assert nonc > 1000
