@@ -52,7 +52,7 @@ static State S;
 constexpr int64_t kRecCap = 1 << 16;  // per-tree statistics kept for gb_tree_stats
 
 static void free_ws(Workspace &w) {
-    void *ptrs[] = {w.visw, w.lvw, w.qv, w.qs, w.qr, w.pkeyq, w.lvl, w.vbase, w.size, w.sz64,
+    void *ptrs[] = {w.vst, w.qv, w.qs, w.qr, w.pkeyq, w.lvl, w.vbase, w.size, w.sz64,
                     w.parq, w.offq, w.szq, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
                     w.scan_tmp};
@@ -90,9 +90,8 @@ static int ensure_workspace(int B, bool descent) {
     Workspace &w = S.ws;
     const Graph &g = S.g;
     const int64_t n = g.n, Bn = (int64_t)B * n, words = (g.m + 31) / 32;
-    const int64_t nw = (n + 31) / 32;
-    ALLOC(w.visw, (int64_t)B * nw);
-    ALLOC(w.lvw, (int64_t)B * 4 * nw);
+    const int64_t nw = (n + 3) / 4;
+    ALLOC(w.vst, (int64_t)B * nw);
     ALLOC(w.qv, Bn);
     ALLOC(w.qs, Bn);
     ALLOC(w.qr, Bn);

@@ -111,8 +111,7 @@ struct Graph {
 struct Workspace {
     int B = 0;                 // capacity in trees
     int64_t n = 0;
-    uint32_t *visw = nullptr;  // [B][n/32] visited bitmap
-    uint32_t *lvw = nullptr;   // [B][4][n/32] level-membership bitmaps (ring of 4)
+    uint32_t *vst = nullptr;   // [B][(n+3)/4] BFS byte states (0 / 0x80 / 0x81 + level mod 127)
     uint32_t *qv = nullptr;    // q: level lists (vertices in BFS level order)
     uint32_t *qs = nullptr;    // q: slot prefix of each queued vertex within its level
     uint32_t *qr = nullptr;    // q: CSR row start of each queued vertex

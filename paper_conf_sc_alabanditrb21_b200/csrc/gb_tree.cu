@@ -6,9 +6,11 @@
 // all B trees advancing level by level inside persistent cooperative kernels
 // (one grid-wide barrier per level for the whole batch, no host round trip).
 //
-// Memory layout: the BFS state of a tree is three
-// bitmaps -- visited, and the membership of levels L-1 / L+1 (a ring of 4) --
-// n/8 bytes each, so the per-slot neighbour tests hit L2.  Everything that is
+// Memory layout: the BFS state of a tree is one
+// byte per vertex (10 MB for a 10M-vertex tree, L2-resident): 0 = unvisited,
+// 0x81 + (level mod 127) = visited at a recent level, 0x80 = visited at least
+// 127 levels ago.  One load answers both per-slot questions (unvisited?  one
+// level up?); discovery is one atomicOr.  Everything that is
 // produced and consumed in BFS order lives in *queue order* (the level lists
 // qv): the parent key, the parent, the sibling offset and the subtree size,
 // so the level passes stream them coalesced.  Only three arrays are indexed
@@ -34,11 +36,11 @@ namespace cg = cooperative_groups;
 struct TreeParams {
     const uint32_t *row_ptr, *adj;
     const int32_t *comp, *coff, *cverts;
-    int64_t n, ncomp, nw;  // nw = bitmap words per tree
+    int64_t n, ncomp, nw;  // nw = state words per tree ((n + 3) / 4)
     int32_t cbig;
     int B;
     int64_t ls;  // stride of lvl / vbase per tree (n + 2)
-    uint32_t *visw, *lvw;  // [B][nw], [B][4][nw]
+    uint32_t *vst;  // [B][nw] byte states, 4 vertices per word
     uint32_t *qv, *qs, *qr;  // qr: row start of each queued vertex
     unsigned long long *pkeyq;
     uint64_t *lvl;
@@ -73,6 +75,9 @@ __device__ __forceinline__ uint32_t warp_incl_scan32(uint32_t v) {
     return v;
 }
 
+// BFS level stamps (see the header comment)
+__device__ __forceinline__ uint32_t level_stamp(int L) { return 0x81u + (uint32_t)(L % 127); }
+
 // parent key of candidate u for w (reading R4): score in the high word, then
 // (u << 1 | neg): the minimum picks the lowest score, ties to the smaller u,
 // and carries the winner's id and the sign of the tree edge
@@ -101,8 +106,7 @@ __global__ void k_batch_prep(TreeParams P) {
 // root of component C in tree b: cverts_C[rkey mod |C|] (reading R4)
 __device__ __forceinline__ void place_root(const TreeParams &P, int b, int64_t C, uint32_t r) {
     const size_t nb = (size_t)b * P.n;
-    atomicOr(P.visw + (size_t)b * P.nw + (r >> 5), 1u << (r & 31));
-    atomicOr(P.lvw + (size_t)b * 4 * P.nw + (r >> 5), 1u << (r & 31));  // level 0
+    atomicOr(P.vst + (size_t)b * P.nw + (r >> 2), level_stamp(0) << (8 * (r & 3)));
     const uint32_t deg = P.row_ptr[r + 1] - P.row_ptr[r];
     const uint32_t pre = (uint32_t)P.coff[C];
     if (deg == 0) {
@@ -192,9 +196,9 @@ __device__ __forceinline__ void expand_range(const TreeParams &P, int b, int L, 
     const uint32_t *qs = P.qs + nb + vb;
     const uint32_t *qv = P.qv + nb + vb;
     const uint32_t *qr = P.qr + nb + vb;
-    uint32_t *visw = P.visw + (size_t)b * P.nw;
-    const uint32_t *lv_prev = P.lvw + ((size_t)b * 4 + ((L + 3) & 3)) * P.nw;
-    uint32_t *lv_next = P.lvw + ((size_t)b * 4 + ((L + 1) & 3)) * P.nw;
+    uint32_t *vst = P.vst + (size_t)b * P.nw;
+    const uint32_t st_prev = level_stamp(L + 126);  // = stamp(L - 1) for L >= 1
+    const uint32_t st_next = level_stamp(L + 1);
     unsigned long long *pk = P.pkeyq + nb + vb;
     // owner of slot s0: the largest q with qs[q] <= s0
     uint32_t q = 0;
@@ -233,26 +237,23 @@ __device__ __forceinline__ void expand_range(const TreeParams &P, int b, int L, 
             const uint32_t a = __ldg(P.adj + j);
             x = a & kIdMask;
             neg = a >> 31;
-            const uint32_t word = x >> 5, bit = 1u << (x & 31);
+            const uint32_t word = x >> 2, sh = 8 * (x & 3);
             if (P.given) {
                 // caller tree: follow tree edges only (parent(x) == w)
                 if (P.given[x] == (int32_t)w) {
                     disc = true;
-                    atomicOr(visw + word, bit);
+                    atomicOr(vst + word, st_next << sh);
                 }
             } else {
-                // both words are independent L2 hits: issue them together
-                const uint32_t vw = __ldcg(visw + word);
-                const uint32_t pw = __ldcg(lv_prev + word);
-                if (!(vw & bit)) {
-                    disc = !(atomicOr(visw + word, bit) & bit);
-                } else if (pw & bit) {
+                const uint32_t st = (__ldcg(vst + word) >> sh) & 0xFFu;
+                if (st == 0) {
+                    disc = !((atomicOr(vst + word, st_next << sh) >> sh) & 0xFFu);
+                } else if (L > 0 && st == st_prev) {
                     // a neighbour one level up is a parent candidate of w (a.3)
                     key = parent_key(tk, x, w, neg);
                 }
             }
             if (disc) {
-                atomicOr(lv_next + word, bit);
                 rs = __ldg(P.row_ptr + x);
                 deg = __ldg(P.row_ptr + x + 1) - rs;
             }
@@ -343,11 +344,17 @@ __global__ void __launch_bounds__(kBlock, 6) k_bfs(TreeParams P) {
             P.lvl[threadIdx.x * P.ls + L + 2] = 0;
             P.vbase[threadIdx.x * P.ls + L + 1] = T.vb[threadIdx.x] + T.nv[threadIdx.x];
         }
-        // clear the level bitmap slot that level L+1 will fill with level L+2
-        // (it held level L-2, read for the last time during level L-1)
-        for (int64_t i = gtid; i < (int64_t)B * P.nw; i += nthr) {
-            const int64_t b = i / P.nw;
-            P.lvw[(b * 4 + ((L + 2) & 3)) * P.nw + (i - b * P.nw)] = 0;
+        // level L+1 compares against stamp(L) == stamp(L-127): retire the
+        // vertices of level L-127 (deep graphs only) so the stamps stay exact
+        if (L >= 127) {
+            for (int b = 0; b < B; b++) {
+                const uint32_t r0 = __ldcg(P.vbase + b * P.ls + (L - 127));
+                const uint32_t r1 = __ldcg(P.vbase + b * P.ls + (L - 126));
+                for (int64_t i = r0 + gtid; i < (int64_t)r1; i += nthr) {
+                    const uint32_t x = __ldcg(P.qv + (size_t)b * P.n + i);
+                    atomicAnd(P.vst + (size_t)b * P.nw + (x >> 2), ~(0x7Fu << (8 * (x & 3))));
+                }
+            }
         }
         __syncthreads();
         const unsigned long long W = T.soff[B];
@@ -634,9 +641,9 @@ static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_
     TreeParams P;
     P.row_ptr = g.row_ptr; P.adj = g.adj;
     P.comp = g.comp; P.coff = g.coff; P.cverts = g.cverts;
-    P.n = g.n; P.ncomp = g.ncomp; P.nw = (g.n + 31) / 32; P.cbig = g.cbig;
+    P.n = g.n; P.ncomp = g.ncomp; P.nw = (g.n + 3) / 4; P.cbig = g.cbig;
     P.B = B; P.ls = g.n + 2;
-    P.visw = ws.visw; P.lvw = ws.lvw; P.qv = ws.qv; P.qs = ws.qs; P.qr = ws.qr; P.pkeyq = ws.pkeyq;
+    P.vst = ws.vst; P.qv = ws.qv; P.qs = ws.qs; P.qr = ws.qr; P.pkeyq = ws.pkeyq;
     P.lvl = ws.lvl; P.vbase = ws.vbase;
     P.size = descent ? nullptr : ws.size;
     P.sz64 = descent ? ws.sz64 : nullptr;
@@ -664,8 +671,7 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
     TreeParams P = make_params(g, ws, B, given_parent, descent);
     const size_t nw = (size_t)P.nw;
     if (ev) GB_CUDA_TRY(cudaEventRecord(ev[0], st));
-    GB_CUDA_TRY(cudaMemsetAsync(ws.visw, 0, sizeof(uint32_t) * (size_t)B * nw, st));
-    GB_CUDA_TRY(cudaMemsetAsync(ws.lvw, 0, sizeof(uint32_t) * (size_t)B * 4 * nw, st));
+    GB_CUDA_TRY(cudaMemsetAsync(ws.vst, 0, sizeof(uint32_t) * (size_t)B * nw, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.s1, 0, sizeof(uint32_t) * (size_t)B * g.ncomp, st));
     if (descent) GB_CUDA_TRY(cudaMemsetAsync(ws.sz64, 0, sizeof(unsigned long long) * (size_t)B * g.n, st));
     else GB_CUDA_TRY(cudaMemsetAsync(ws.size, 0, sizeof(uint32_t) * (size_t)B * g.n, st));
