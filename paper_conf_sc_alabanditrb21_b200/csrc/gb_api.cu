@@ -188,11 +188,9 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     const int64_t K = t_end > t_begin ? (t_end - t_begin + stride - 1) / stride : 0;
     if (K == 0) return GB_OK;
     const bool descent = S.opt.walk == 1;
-    if (descent && (int64_t)kMaxBatch * S.g.n >= (1ll << 32)) {
-        set_error("walk=1 needs batch*n < 2^32");
-        return GB_EINVAL;
-    }
-    const int B = auto_batch(K);
+    int B = auto_batch(K);
+    // walk 1 keeps child lists of a whole batch in one 32-bit index space
+    if (descent) B = (int)std::min<int64_t>(B, std::max<int64_t>(1, ((1ll << 32) - 1) / S.g.n));
     int rc = ensure_workspace(B, descent);
     if (rc) return rc;
     const int G = auto_group(B);

@@ -13,7 +13,7 @@ constexpr uint32_t kNegBit = 0x80000000u;   // sign bit packed next to a 31-bit 
 constexpr uint32_t kIdMask = 0x7FFFFFFFu;
 constexpr int32_t kInf = 0x7F7F7F7F;         // "unvisited" BFS distance (memset 0x7F)
 constexpr uint32_t kNone = 0xFFFFFFFFu;
-constexpr int kMaxBatch = 64;                // trees per batch (smem tables)
+constexpr int kMaxBatch = 128;               // trees per batch (smem tables)
 constexpr int kBlock = 256;                  // threads per CTA of the cooperative kernels
 
 // ---------------------------------------------------------------------------
