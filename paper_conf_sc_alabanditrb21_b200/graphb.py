@@ -41,10 +41,11 @@ def lib():
     global _lib
     if _lib is not None:
         return _lib
-    if not os.path.exists(_build.LIB):
-        raise RuntimeError(f"{_build.LIB} is missing: run __graft_entry__.build() "
+    path = os.environ.get("GRAPHB_LIB", _build.LIB)   # alternative in-tree builds (experiments)
+    if not os.path.exists(path):
+        raise RuntimeError(f"{path} is missing: run __graft_entry__.build() "
                            "(the CUDA library is required; there is no fallback)")
-    L = ctypes.CDLL(_build.LIB)
+    L = ctypes.CDLL(path)
     P, i64, u64, i32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_uint64, ctypes.c_int
     sig = {
         "gb_load_csr": (i32, [i64, i64, P, P, P]),
