@@ -115,8 +115,12 @@ int gb_set_option(const char *key, int64_t value);
 int gb_get_stats(int64_t *ints, int n_ints, double *phase_ms, int n_phase);
 
 /* Per-tree statistics of the last gb_balance* call, for at most max_trees
- * trees in processing order: out[3*i] = sum of cycle lengths, out[3*i+1] =
- * cycles, out[3*i+2] = depth; tree_ids[i] = t.  Returns the count. */
+ * (<= 65536 recorded) trees in processing order: out[4*i] = sum of cycle
+ * lengths, out[4*i+1] = cycles, out[4*i+2] = depth, out[4*i+3] = signature of
+ * the tree's nearest balanced state (XOR over switched eids e of
+ * mix64(e ^ 0x5851F42D4C957F2D); equal states <=> equal signatures up to
+ * 2^-64 collisions -- frustration-cloud analytics, Fig. 2 L81/L86);
+ * tree_ids[i] = t.  Returns the count. */
 int64_t gb_tree_stats(uint64_t *out, int64_t *tree_ids, int64_t max_trees);
 
 /* Ingest results (§8 a.1), copied to host arrays (any pointer may be NULL):

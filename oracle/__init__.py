@@ -63,6 +63,8 @@ def lib():
                                       ctypes.POINTER(ctypes.c_int32)]
         L.or_preorder.restype = ctypes.c_int; L.or_preorder.argtypes = [P, P, P, P]
         L.or_harary.restype = ctypes.c_int; L.or_harary.argtypes = [P, P, P, P]
+        L.or_state_signature.restype = u64
+        L.or_state_signature.argtypes = [P, i64]
         L.or_balance.restype = ctypes.c_int
         L.or_balance.argtypes = [P, i64, i64, i64, u64, P, P, P]
         _lib = L
@@ -96,6 +98,11 @@ def ekey(seed, t, e):
 
 def pscore(seed, t, a, b):
     return int(lib().or_pscore(seed, t, a, b))
+
+
+def state_signature(flip):
+    flip = np.ascontiguousarray(flip, dtype=np.uint8)
+    return int(lib().or_state_signature(_p(flip) if len(flip) else None, len(flip)))
 
 
 class OracleError(RuntimeError):
@@ -183,11 +190,11 @@ class Graph:
         """Frustration cloud over trees t_begin, t_begin+stride, ... < num_trees."""
         cnt = np.zeros(max(self.m, 1), np.uint32); agree = np.zeros(self.n, np.uint32)
         k = len(range(t_begin, num_trees, stride))
-        stats = np.zeros(3 * max(k, 1), np.uint64)
+        stats = np.zeros(4 * max(k, 1), np.uint64)
         rc = lib().or_balance(self._h, t_begin, num_trees, stride, seed, _p(cnt), _p(agree),
                               _p(stats))
         if rc != OR_OK:
             raise OracleError(rc, "or_balance")
         if with_stats:
-            return cnt[: self.m], agree, stats[: 3 * k].reshape(k, 3)
+            return cnt[: self.m], agree, stats[: 4 * k].reshape(k, 4)
         return cnt[: self.m], agree

@@ -504,6 +504,21 @@ out:
 }
 
 /* ------------------------------------------------------------------------ */
+/* Frustration-cloud analytics (Fig. 2 L81/L86: the cloud is
+ * the set of *unique* nearest balanced states).  A balanced state Sigma_T is
+ * identified by its switch set; its signature is the XOR over switched edges
+ * e of mix64(e XOR 0x5851F42D4C957F2D).  Equal states have equal signatures;
+ * distinct states collide with probability 2^-64.                           */
+/* ------------------------------------------------------------------------ */
+uint64_t or_state_signature(const uint8_t *flip, int64_t m)
+{
+    uint64_t s = 0;
+    for (int64_t e = 0; e < m; e++)
+        if (flip[e]) s ^= or_mix64((uint64_t)e ^ 0x5851F42D4C957F2DULL);
+    return s;
+}
+
+/* ------------------------------------------------------------------------ */
 /* Alg. 2 (L125-L138) over the trees t_begin, t_begin+stride, ... < t_end:
  * sample T (BFS), balance (Alg. 1), Harary bipartition (L224), count per
  * edge and per vertex (L248).                                               */
@@ -533,7 +548,12 @@ int or_balance(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride
         if (rc != OR_OK) goto out;
         for (int64_t e = 0; e < m; e++) cnt[e] += flip[e];
         for (int64_t v = 0; v < n; v++) agree[v] += delta2[v];
-        if (stats) { stats[3 * i] = sk; stats[3 * i + 1] = (uint64_t)nc; stats[3 * i + 2] = (uint64_t)md; }
+        if (stats) {
+            stats[4 * i] = sk;
+            stats[4 * i + 1] = (uint64_t)nc;
+            stats[4 * i + 2] = (uint64_t)md;
+            stats[4 * i + 3] = or_state_signature(flip, m);
+        }
     }
     rc = OR_OK;
 out:

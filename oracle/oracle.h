@@ -63,9 +63,13 @@ int or_preorder(const or_graph *g, const int32_t *parent, int32_t *pre, int32_t 
  * (L144: 2 larger side, 1 tie, 0 smaller side), per connected component. */
 int or_harary(const or_graph *g, const uint8_t *flip, uint8_t *side, uint8_t *delta2);
 
+/* Signature of the nearest balanced state with switch set flip[0..m)
+ * (SURVEY §8 f.2): XOR over switched e of mix64(e ^ 0x5851F42D4C957F2D). */
+uint64_t or_state_signature(const uint8_t *flip, int64_t m);
+
 /* --- frustration cloud (Alg. 2 over trees t_begin, t_begin+stride, ... < t_end)
  * cnt[e] += flip_t(e); agree[v] += delta2_t(v);
- * stats (may be NULL): per processed tree {sumk, ncyc, maxdepth}. */
+ * stats (may be NULL): per processed tree {sumk, ncyc, maxdepth, state signature}. */
 int or_balance(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride,
                uint64_t seed, uint32_t *cnt, uint32_t *agree, uint64_t *stats);
 

@@ -30,7 +30,7 @@ struct Stats {
     uint64_t sumk = 0, cycles = 0;
     int64_t max_depth = 0;
     double phase_ms[GB_NPHASE] = {0};
-    std::vector<uint64_t> per_tree;   // 3 per recorded tree
+    std::vector<uint64_t> per_tree;   // 4 per recorded tree
     std::vector<int64_t> tree_ids;
 };
 
@@ -43,7 +43,7 @@ struct State {
     int32_t *d_cnt = nullptr, *d_agree = nullptr;  // gb_balance's device counters
     int32_t *d_given = nullptr;                    // caller tree (gb_balance_given_tree)
     unsigned long long *d_visited = nullptr;       // [kMaxBatch]
-    unsigned long long *d_rec_stats = nullptr;     // [kRecCap][3]
+    unsigned long long *d_rec_stats = nullptr;     // [kRecCap][4]
     std::vector<int32_t> h_comp;
     Options opt;
     Stats st;
@@ -107,7 +107,7 @@ static int ensure_workspace(int B, bool descent) {
     ALLOC(w.s1, (int64_t)B * g.ncomp);
     ALLOC(w.tkey, kMaxBatch);
     ALLOC(w.depth, kMaxBatch);
-    ALLOC(w.tstat, 2 * kMaxBatch);
+    ALLOC(w.tstat, 3 * kMaxBatch);
     ALLOC(w.visited, kMaxBatch);
     ALLOC(w.maxd, 1);
     if (descent) {
@@ -154,9 +154,10 @@ __global__ void k_record_stats(const unsigned long long *tstat, const int32_t *d
                                unsigned long long *rec, int64_t pos, int64_t cap) {
     int b = threadIdx.x;
     if (b < B && pos + b < cap) {
-        rec[3 * (pos + b)] = tstat[2 * b];
-        rec[3 * (pos + b) + 1] = tstat[2 * b + 1];
-        rec[3 * (pos + b) + 2] = (unsigned long long)depth[b];
+        rec[4 * (pos + b)] = tstat[3 * b];
+        rec[4 * (pos + b) + 1] = tstat[3 * b + 1];
+        rec[4 * (pos + b) + 2] = (unsigned long long)depth[b];
+        rec[4 * (pos + b) + 3] = tstat[3 * b + 2];
     }
 }
 
@@ -197,7 +198,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     T.batch_used = B;
     T.group_used = G;
     if (!S.d_rec_stats) {
-        GB_CUDA_TRY(cudaMalloc(&S.d_rec_stats, sizeof(unsigned long long) * 3 * kRecCap));
+        GB_CUDA_TRY(cudaMalloc(&S.d_rec_stats, sizeof(unsigned long long) * 4 * kRecCap));
     }
     std::vector<cudaEvent_t> evs;
     const bool timing = S.opt.timing != 0;
@@ -214,7 +215,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         }
         k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, nb, seed, t0, stride);
         ++T.launches;
-        GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 2 * nb, st));
+        GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 3 * nb, st));
         rc = run_batch_tree(S.g, S.ws, nb, nullptr, st, &T.launches, ev, descent);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
@@ -234,15 +235,15 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     }
     GB_CUDA_TRY(cudaGetLastError());
     const int64_t nrec = std::min<int64_t>(K, kRecCap);
-    T.per_tree.resize(3 * nrec);
-    GB_CUDA_TRY(cudaMemcpyAsync(T.per_tree.data(), S.d_rec_stats, sizeof(uint64_t) * 3 * nrec,
+    T.per_tree.resize(4 * nrec);
+    GB_CUDA_TRY(cudaMemcpyAsync(T.per_tree.data(), S.d_rec_stats, sizeof(uint64_t) * 4 * nrec,
                                 cudaMemcpyDeviceToHost, st));
     GB_CUDA_TRY(cudaStreamSynchronize(st));
     T.trees = K;
     for (int64_t i = 0; i < nrec; i++) {
-        T.sumk += T.per_tree[3 * i];
-        T.cycles += T.per_tree[3 * i + 1];
-        T.max_depth = std::max<int64_t>(T.max_depth, (int64_t)T.per_tree[3 * i + 2]);
+        T.sumk += T.per_tree[4 * i];
+        T.cycles += T.per_tree[4 * i + 1];
+        T.max_depth = std::max<int64_t>(T.max_depth, (int64_t)T.per_tree[4 * i + 2]);
     }
     if (timing) {
         for (size_t base = 0; base < evs.size(); base += GB_NPHASE + 1) {
@@ -265,7 +266,7 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
     cudaStream_t st = S.stream;
     k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, 1, seed, t, 1);
     ++T.launches;
-    GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 2, st));
+    GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 3, st));
     rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk == 1);
     if (rc) return rc;
     if (d_given) {
@@ -506,7 +507,7 @@ int64_t gb_tree_stats(uint64_t *out, int64_t *tree_ids, int64_t max_trees) {
     const Stats &T = S.st;
     int64_t k = std::min<int64_t>(max_trees, (int64_t)T.tree_ids.size());
     for (int64_t i = 0; i < k; i++) {
-        if (out) for (int j = 0; j < 3; j++) out[3 * i + j] = T.per_tree[3 * i + j];
+        if (out) for (int j = 0; j < 4; j++) out[4 * i + j] = T.per_tree[4 * i + j];
         if (tree_ids) tree_ids[i] = T.tree_ids[i];
     }
     return k;

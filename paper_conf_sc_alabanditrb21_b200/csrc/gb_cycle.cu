@@ -37,7 +37,7 @@ struct CycleParams {
     const uint2 *crec;     // [B][n] pre-indexed {child-list start, #children}
     const uint32_t *clist; // children pre IDs, per parent ascending
     uint32_t *fbits;       // [B][words]
-    unsigned long long *tstat;  // [B][2]
+    unsigned long long *tstat;  // [B][3] {sum cycle length, cycles, state signature}
     int64_t words;
     int b0, G;             // trees b0 .. b0+G-1 of the batch
 };
@@ -45,14 +45,51 @@ struct CycleParams {
 constexpr int kCycleBlock = 256;
 constexpr int kMaxGroup = 64;
 
+// f.2: signature of a nearest balanced state = XOR over its switched edges of
+// mix64(e ^ K) (order-free, so each warp reduces its 32 edges on its own)
+constexpr uint64_t kSigSalt = 0x5851F42D4C957F2Dull;
+
+__device__ __forceinline__ void warp_stats(int lane, int g, uint32_t k, bool cyc, bool flip,
+                                           int64_t e, unsigned long long *s_k,
+                                           unsigned long long *s_c, unsigned long long *s_sig) {
+    uint32_t kk = k, cc = cyc ? 1u : 0u;
+    unsigned long long sig = flip ? mix64((uint64_t)e ^ kSigSalt) : 0ull;
+#pragma unroll
+    for (int d = 16; d; d >>= 1) {
+        kk += __shfl_xor_sync(0xFFFFFFFFu, kk, d);
+        cc += __shfl_xor_sync(0xFFFFFFFFu, cc, d);
+        sig ^= __shfl_xor_sync(0xFFFFFFFFu, sig, d);
+    }
+    if (lane == 0) {
+        if (cc) {
+            atomicAdd(&s_k[g], (unsigned long long)kk);
+            atomicAdd(&s_c[g], (unsigned long long)cc);
+        }
+        if (sig) atomicXor(&s_sig[g], sig);
+    }
+}
+
+__device__ __forceinline__ void flush_stats(const CycleParams &P, const unsigned long long *s_k,
+                                            const unsigned long long *s_c,
+                                            const unsigned long long *s_sig) {
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) {
+        unsigned long long *t = P.tstat + 3 * (P.b0 + i);
+        if (s_c[i]) {
+            atomicAdd(t, s_k[i]);
+            atomicAdd(t + 1, s_c[i]);
+        }
+        if (s_sig[i]) atomicXor(t + 2, s_sig[i]);
+    }
+}
+
 __device__ __forceinline__ bool is_anc(uint32_t a, uint32_t size_a, uint32_t t) {
     return (t - a) < size_a;  // a <= t <= a + size_a - 1 (unsigned wrap for t < a)
 }
 
 // one warp = 32 consecutive edges (one flip word per tree)
 __global__ void __launch_bounds__(kCycleBlock) k_cycles_two_ended(CycleParams P) {
-    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup];
-    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; }
+    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup], s_sig[kMaxGroup];
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; s_sig[i] = 0; }
     __syncthreads();
     const int lane = threadIdx.x & 31;
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -98,33 +135,19 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_two_ended(CycleParams P)
             }
             const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
             if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
-            // per-tree cycle statistics (warp reduce, then shared atomics)
-            uint32_t kk = k, cc = cyc ? 1u : 0u;
-#pragma unroll
-            for (int d = 16; d; d >>= 1) {
-                kk += __shfl_xor_sync(0xFFFFFFFFu, kk, d);
-                cc += __shfl_xor_sync(0xFFFFFFFFu, cc, d);
-            }
-            if (lane == 0 && cc) {
-                atomicAdd(&s_k[g], (unsigned long long)kk);
-                atomicAdd(&s_c[g], (unsigned long long)cc);
-            }
+            // per-tree cycle statistics and state signature
+            warp_stats(lane, g, k, cyc, flip != 0, e, s_k, s_c, s_sig);
         }
     }
     __syncthreads();
-    for (int i = threadIdx.x; i < P.G; i += blockDim.x) {
-        if (s_c[i]) {
-            atomicAdd(P.tstat + 2 * (P.b0 + i), s_k[i]);
-            atomicAdd(P.tstat + 2 * (P.b0 + i) + 1, s_c[i]);
-        }
-    }
+    flush_stats(P, s_k, s_c, s_sig);
 }
 
 // Alg. 3 as written: lane-parallel climb to the LCA, then warp-cooperative
 // descents from the LCA to v, one lane's cycle at a time.
 __global__ void __launch_bounds__(kCycleBlock) k_cycles_descent(CycleParams P) {
-    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup];
-    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; }
+    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup], s_sig[kMaxGroup];
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; s_sig[i] = 0; }
     __syncthreads();
     const int lane = threadIdx.x & 31;
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -193,25 +216,11 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_descent(CycleParams P) {
             const uint32_t flip = cyc ? ((c >> 31) ^ nege) : 0u;
             const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
             if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
-            uint32_t kk = k, cc = cyc ? 1u : 0u;
-#pragma unroll
-            for (int d = 16; d; d >>= 1) {
-                kk += __shfl_xor_sync(0xFFFFFFFFu, kk, d);
-                cc += __shfl_xor_sync(0xFFFFFFFFu, cc, d);
-            }
-            if (lane == 0 && cc) {
-                atomicAdd(&s_k[g], (unsigned long long)kk);
-                atomicAdd(&s_c[g], (unsigned long long)cc);
-            }
+            warp_stats(lane, g, k, cyc, flip != 0, e, s_k, s_c, s_sig);
         }
     }
     __syncthreads();
-    for (int i = threadIdx.x; i < P.G; i += blockDim.x) {
-        if (s_c[i]) {
-            atomicAdd(P.tstat + 2 * (P.b0 + i), s_k[i]);
-            atomicAdd(P.tstat + 2 * (P.b0 + i) + 1, s_c[i]);
-        }
-    }
+    flush_stats(P, s_k, s_c, s_sig);
 }
 
 // ---------------------------------------------------------------------------

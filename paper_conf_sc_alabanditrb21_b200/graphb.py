@@ -240,7 +240,18 @@ def stats():
 
 
 def tree_stats(max_trees=1 << 16):
-    out = np.zeros(3 * max_trees, np.uint64)
+    """Per-tree (sum of cycle lengths, cycles, depth, state signature) of the
+    last balance call."""
+    out = np.zeros(4 * max_trees, np.uint64)
     ids = np.zeros(max_trees, np.int64)
     k = lib().gb_tree_stats(_ptr(out), _ptr(ids), max_trees)
-    return ids[:k], out[: 3 * k].reshape(k, 3)
+    return ids[:k], out[: 4 * k].reshape(k, 4)
+
+
+def cloud_states(max_trees=1 << 16):
+    """Frustration-cloud analytics of the last balance call:
+    {state signature: number of sampled trees reaching that nearest balanced
+    state}.  len() of it is the number of distinct states found."""
+    _, per = tree_stats(max_trees)
+    sigs, counts = np.unique(per[:, 3], return_counts=True)
+    return {int(s): int(c) for s, c in zip(sigs, counts)}

@@ -38,6 +38,7 @@ def check_cloud(g, T, seed, **opts):
     assert np.array_equal(per[:, 0], ostats[:, 0]), "per-tree sum of cycle lengths"
     assert np.array_equal(per[:, 1], ostats[:, 1]), "per-tree cycles"
     assert np.array_equal(per[:, 2], ostats[:, 2]), "per-tree depth"
+    assert np.array_equal(per[:, 3], ostats[:, 3]), "per-tree state signature (f.2)"
     assert st["cycles"] == T * (g.m - g.n + og.ncomp)     # L112
     return st
 
@@ -102,6 +103,19 @@ def test_power_law_hubs_multi_batch(walk):
     """Hubs (Chung-Lu) + several batches + cycle groups smaller than a batch."""
     g = graphgen.chung_lu(20000, 90000, 2500, 0.75, 0.25, 3)
     check_cloud(g, 37, 11, batch=16, cycle_group=5, walk=walk)
+
+
+def test_frustration_cloud_distinct_states():
+    """f.2 (Fig. 2, L81/L86): distinct nearest balanced states over many
+    trees, counted from the per-tree state signatures, equal the oracle's."""
+    g = graphgen.random_tiny(7, 11, 0.4, seed=3)
+    check_cloud(g, 200, 5)
+    states = graphb.cloud_states()
+    og = oracle.Graph.from_csr(g)
+    _, _, ostats = og.balance(200, 5, with_stats=True)
+    assert len(states) == len(set(int(x) for x in ostats[:, 3]))
+    assert sum(states.values()) == 200
+    assert len(states) > 1
 
 
 def test_disconnected_forest_with_isolated_vertices():

@@ -445,6 +445,13 @@ def test_diamond_frustration_cloud():
         _, d2 = og.harary(flip)
         agree += d2
     assert len(states) == int(facts["unique_states"][0])          # L81, L86
+    # f.2: the state signature separates exactly the distinct states
+    sigs = {}
+    for tree in trees:
+        parent = bf.parent_array(g.n, tree, [0])
+        flip, _, _, _ = og.balance_tree(np.array(parent, np.int32))
+        sigs.setdefault(oracle.state_signature(flip), set()).add(tuple(flip.tolist()))
+    assert len(sigs) == len(states) and all(len(v) == 1 for v in sigs.values())
     assert max(states.values()) == int(facts["top_state_count"][0])  # L112
     assert states[tuple([0] * g.m)] == int(facts["top_state_count"][0])  # all-positive state
     assert agree.tolist() == [int(x) for x in facts["agree"]]     # L144 (6/8)
@@ -472,6 +479,17 @@ def test_oracle_rejects_invalid_csr():
     for rp, c, s in bad:
         with pytest.raises(oracle.OracleError):
             oracle.Graph(rp, c, s)
+
+
+def test_state_signature_definition():
+    """f.2 signature: XOR-linear over switched edges, empty set -> 0."""
+    assert oracle.state_signature(np.zeros(5, np.uint8)) == 0
+    a = np.array([1, 0, 1, 0, 0], np.uint8)
+    b = np.array([0, 0, 1, 1, 0], np.uint8)
+    ab = a ^ b
+    assert oracle.state_signature(a) ^ oracle.state_signature(b) == oracle.state_signature(ab)
+    one = np.array([0, 0, 0, 1], np.uint8)
+    assert oracle.state_signature(one) == oracle.mix64(3 ^ 0x5851F42D4C957F2D)
 
 
 def test_tree_sharding_is_additive():
