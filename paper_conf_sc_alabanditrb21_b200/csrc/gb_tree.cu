@@ -536,6 +536,49 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
     for (int L = 0; L <= maxd; L++) {
         load_level(P, L, T, s_depth);
         const unsigned long long total = T.soff[B];
+        if (!kDescent && L > 0) {
+            // kILP independent vertices per thread per iteration: their queue
+            // words, then their parents' labels, are in flight together
+            constexpr int kILP = 4;
+            for (unsigned long long base = gtid; base < total; base += kILP * nthr) {
+                size_t qi[kILP], nbk[kILP];
+                uint32_t x[kILP], pq[kILP], off[kILP], szx[kILP], ppp[kILP];
+                int bk[kILP];
+#pragma unroll
+                for (int k = 0; k < kILP; k++) {
+                    const unsigned long long i = base + (unsigned long long)k * nthr;
+                    bk[k] = -1;
+                    if (i < total) {
+                        bk[k] = tree_of(T, B, i);
+                        nbk[k] = (size_t)bk[k] * P.n;
+                        qi[k] = nbk[k] + T.vb[bk[k]] + (uint32_t)(i - T.soff[bk[k]]);
+                        x[k] = __ldcg(P.qv + qi[k]);
+                        pq[k] = __ldcg(P.parq + qi[k]);
+                        off[k] = __ldcg(P.offq + qi[k]);
+                        szx[k] = __ldcg(P.szq + qi[k]);
+                    }
+                }
+#pragma unroll
+                for (int k = 0; k < kILP; k++)
+                    if (bk[k] >= 0) ppp[k] = __ldcg(P.pp + nbk[k] + (pq[k] & kIdMask));
+#pragma unroll
+                for (int k = 0; k < kILP; k++) {
+                    if (bk[k] < 0) continue;
+                    const uint32_t up = ppp[k] & kIdMask, neg = pq[k] & kNegBit;
+                    const uint32_t pre = up + off[k];
+                    const uint32_t pi = (ppp[k] & kNegBit) ^ neg;
+                    P.pp[nbk[k] + x[k]] = pre | pi;
+                    P.rec[nbk[k] + pre] = make_uint2(up | neg, szx[k]);
+                    if (pi) {
+                        const int32_t C = one_comp ? 0 : __ldg(P.comp + x[k]);
+                        if (C == P.cbig) atomicAdd(&s_big[bk[k]], 1u);
+                        else atomicAdd(P.s1 + (size_t)bk[k] * P.ncomp + C, 1u);
+                    }
+                }
+            }
+            grid.sync();
+            continue;
+        }
         for (unsigned long long i = gtid; i < total; i += nthr) {
             const int b = tree_of(T, B, i);
             const size_t nb = (size_t)b * P.n;
