@@ -82,6 +82,17 @@ class ClockSampler:
     def stop(self):
         if self.proc is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        if not self.lines:
+            # timed region shorter than the sampling period: one sample right after it
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.FIELDS}",
+                                      "--format=csv,noheader,nounits"], capture_output=True,
+                                     text=True, timeout=10).stdout.strip()
+                if out:
+                    self.lines.append(out.splitlines()[0])
+                    self.post = True
+            except Exception:
+                pass
         self.proc.terminate()
         try:
             self.proc.wait(timeout=5)
@@ -102,9 +113,12 @@ class ClockSampler:
             for nm, val in zip(names, p[3:7]):
                 if val.lower().startswith("active"):
                     reasons.add(nm)
-        return {"sm_mhz": statistics.median(sm) if sm else None,
-                "sm_max_mhz": max(smax) if smax else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+        out = {"sm_mhz": statistics.median(sm) if sm else None,
+               "sm_max_mhz": max(smax) if smax else None,
+               "reasons": sorted(reasons), "samples": len(sm)}
+        if getattr(self, "post", False):
+            out["note"] = "timed region shorter than 100 ms: one sample taken right after it"
+        return out
 
 
 # ---------------------------------------------------------------------------

@@ -18,6 +18,33 @@ namespace gb {
 static std::string g_err;
 void set_error(const std::string &msg) { g_err = msg; }
 
+static void *g_arena[kArSlots] = {nullptr};
+static size_t g_arena_cap[kArSlots] = {0};
+
+void *arena(int slot, size_t bytes) {
+    bytes = std::max<size_t>(bytes, 256);
+    if (g_arena_cap[slot] >= bytes) return g_arena[slot];
+    if (g_arena[slot]) cudaFree(g_arena[slot]);
+    g_arena[slot] = nullptr;
+    g_arena_cap[slot] = 0;
+    cudaError_t e = cudaMalloc(&g_arena[slot], bytes);
+    if (e != cudaSuccess) {
+        set_error(std::string("cudaMalloc (graph buffers): ") + cudaGetErrorString(e));
+        g_arena[slot] = nullptr;
+        return nullptr;
+    }
+    g_arena_cap[slot] = bytes;
+    return g_arena[slot];
+}
+
+void arena_free_all() {
+    for (int i = 0; i < kArSlots; i++) {
+        if (g_arena[i]) cudaFree(g_arena[i]);
+        g_arena[i] = nullptr;
+        g_arena_cap[i] = 0;
+    }
+}
+
 struct Options {
     int64_t batch = 0;       // 0 = auto
     int64_t cycle_group = 0; // 0 = auto
@@ -45,6 +72,7 @@ struct State {
     unsigned long long *d_visited = nullptr;       // [kMaxBatch]
     unsigned long long *d_rec_stats = nullptr;     // [kRecCap][4]
     std::vector<int32_t> h_comp;
+    size_t free_at_load = 0;   // device memory free after ingest (cudaMemGetInfo costs ~2 ms)
     Options opt;
     Stats st;
 };
@@ -61,9 +89,7 @@ static void free_ws(Workspace &w) {
 }
 
 static void free_graph(Graph &g) {
-    void *ptrs[] = {g.row_ptr, g.adj, g.adj_eid, g.edges, g.comp, g.coff, g.cverts};
-    for (void *p : ptrs) if (p) cudaFree(p);
-    g = Graph();
+    g = Graph();   // the arrays live in the persistent arena
 }
 
 static size_t per_tree_bytes(const Graph &g, bool descent) {
@@ -163,9 +189,7 @@ __global__ void k_record_stats(const unsigned long long *tstat, const int32_t *d
 
 static int auto_batch(int64_t ntrees) {
     if (S.opt.batch > 0) return (int)std::min<int64_t>(S.opt.batch, kMaxBatch);
-    size_t freeb = 0, totb = 0;
-    cudaMemGetInfo(&freeb, &totb);
-    size_t have = freeb + (size_t)S.ws.B * per_tree_bytes(S.g, S.ws_descent);
+    const size_t have = S.free_at_load;
     int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk == 1));
     int64_t b = std::min<int64_t>({ntrees, (int64_t)kMaxBatch, std::max<int64_t>(bm, 1)});
     // large graphs: a few trees per batch already fill the GPU
@@ -324,14 +348,23 @@ int gb_selftest(void) {
     return GB_OK;
 }
 
-void gb_free(void) {
-    if (S.loaded || S.ws.B) {
-        free_ws(S.ws);
-        free_graph(S.g);
-    }
+// release the loaded graph and everything sized by it, but keep the stream,
+// the statistics buffer and (if asked) the tree workspace for a reload
+static void release_graph(bool keep_ws) {
+    if (!keep_ws) free_ws(S.ws);
+    free_graph(S.g);
     if (S.d_cnt) cudaFree(S.d_cnt);
     if (S.d_agree) cudaFree(S.d_agree);
     if (S.d_given) cudaFree(S.d_given);
+    S.d_cnt = S.d_agree = nullptr;
+    S.d_given = nullptr;
+    S.loaded = false;
+    S.h_comp.clear();
+}
+
+void gb_free(void) {
+    release_graph(false);
+    arena_free_all();
     if (S.d_visited) cudaFree(S.d_visited);
     if (S.d_rec_stats) cudaFree(S.d_rec_stats);
     if (S.stream) cudaStreamDestroy(S.stream);
@@ -351,20 +384,30 @@ int gb_load_csr(int64_t n, int64_t m, const int64_t *row_ptr, const int32_t *col
     }
     int rc = check_device();
     if (rc) return rc;
-    gb_free();
     int dev = 0;
     GB_CUDA_TRY(cudaGetDevice(&dev));
+    // a reload on the same device keeps the tree workspace if the new graph
+    // has the same shape (all dynamic memory allocated once, L236)
+    const bool same_dev = S.stream != nullptr && S.g.dev == dev;
+    const int64_t old_n = S.g.n, old_m = S.g.m, old_c = S.g.ncomp;
+    if (same_dev) release_graph(true); else gb_free();
     int coop = 0;
     GB_CUDA_TRY(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev));
     if (!coop) { set_error("device lacks cooperative launch"); return GB_ECUDA; }
     S.g.dev = dev;
     GB_CUDA_TRY(cudaDeviceGetAttribute(&S.g.num_sms, cudaDevAttrMultiProcessorCount, dev));
-    GB_CUDA_TRY(cudaStreamCreateWithFlags(&S.stream, cudaStreamNonBlocking));
+    if (!S.stream) GB_CUDA_TRY(cudaStreamCreateWithFlags(&S.stream, cudaStreamNonBlocking));
     int64_t launches = 0;
     rc = ingest(S.g, n, m, row_ptr, col_idx, sign, S.stream, &launches);
     if (rc) { gb_free(); return rc; }
+    if (S.ws.B && (S.g.n != old_n || S.g.m != old_m || S.g.ncomp != old_c)) free_ws(S.ws);
     S.h_comp.resize(n);
     GB_CUDA_TRY(cudaMemcpy(S.h_comp.data(), S.g.comp, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+    {
+        size_t freeb = 0, totb = 0;
+        GB_CUDA_TRY(cudaMemGetInfo(&freeb, &totb));
+        S.free_at_load = freeb + (size_t)S.ws.B * per_tree_bytes(S.g, S.ws_descent);
+    }
     S.loaded = true;
     S.st = Stats();
     S.st.launches = launches;

@@ -310,23 +310,28 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
             goto done;                                                         \
         }                                                                      \
     } while (0)
-    ING_TRY(cudaMalloc(&d_rp64, sizeof(int64_t) * (n + 1)));
-    ING_TRY(cudaMalloc(&d_col, sizeof(int32_t) * std::max<uint64_t>(slots, 1)));
-    ING_TRY(cudaMalloc(&d_sign, std::max<uint64_t>(slots, 1)));
-    ING_TRY(cudaMalloc(&d_err, sizeof(uint32_t)));
-    ING_TRY(cudaMalloc(&g.row_ptr, sizeof(uint32_t) * (n + 1)));
-    ING_TRY(cudaMalloc(&g.adj, sizeof(uint32_t) * std::max<uint64_t>(slots, 1)));
-    ING_TRY(cudaMalloc(&g.adj_eid, sizeof(uint32_t) * std::max<uint64_t>(slots, 1)));
-    ING_TRY(cudaMalloc(&g.edges, sizeof(uint2) * std::max<int64_t>(m, 1)));
-    ING_TRY(cudaMalloc(&g.comp, sizeof(int32_t) * n));
-    ING_TRY(cudaMalloc(&g.cverts, sizeof(int32_t) * n));
-    ING_TRY(cudaMalloc(&uptr, sizeof(uint32_t) * n));
-    ING_TRY(cudaMalloc(&upc, sizeof(uint32_t) * n));
-    ING_TRY(cudaMalloc(&ebase, sizeof(uint32_t) * n));
-    ING_TRY(cudaMalloc(&tmp, sizeof(uint32_t) * ntmp));
-    ING_TRY(cudaMalloc(&lab, sizeof(int32_t) * n));
-    ING_TRY(cudaMalloc(&flag, sizeof(uint32_t) * n));
-    ING_TRY(cudaMalloc(&rank, sizeof(uint32_t) * n));
+#define ING_ALLOC(ptr, slot, count)                                                         \
+    do {                                                                                    \
+        ptr = (decltype(ptr))arena(slot, sizeof(*ptr) * (size_t)std::max<uint64_t>((uint64_t)(count), 1)); \
+        if (!ptr) { fail(GB_ENOMEM); goto done; }                                          \
+    } while (0)
+    ING_ALLOC(d_rp64, kArRowPtr64, n + 1);
+    ING_ALLOC(d_col, kArCol, slots);
+    ING_ALLOC(d_sign, kArSign, slots);
+    ING_ALLOC(d_err, kArErr, 1);
+    ING_ALLOC(g.row_ptr, kArRowPtr, n + 1);
+    ING_ALLOC(g.adj, kArAdj, slots);
+    ING_ALLOC(g.adj_eid, kArAdjEid, slots);
+    ING_ALLOC(g.edges, kArEdges, m);
+    ING_ALLOC(g.comp, kArComp, n);
+    ING_ALLOC(g.cverts, kArCverts, n);
+    ING_ALLOC(uptr, kArUptr, n);
+    ING_ALLOC(upc, kArUpc, n);
+    ING_ALLOC(ebase, kArEbase, n);
+    ING_ALLOC(tmp, kArScanTmp, ntmp);
+    ING_ALLOC(lab, kArLab, n);
+    ING_ALLOC(flag, kArFlag, n);
+    ING_ALLOC(rank, kArRank, n);
     ING_TRY(cudaMemcpyAsync(d_rp64, h_row_ptr, sizeof(int64_t) * (n + 1), cudaMemcpyHostToDevice, st));
     if (slots) {
         ING_TRY(cudaMemcpyAsync(d_col, h_col, sizeof(int32_t) * slots, cudaMemcpyHostToDevice, st));
@@ -381,7 +386,7 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
         for (int64_t v = 0; v < n; v++) cv[fill[hc[v]]++] = (int32_t)v;
         g.ncomp = nc;
         g.cbig = big;
-        ING_TRY(cudaMalloc(&g.coff, sizeof(int32_t) * (nc + 1)));
+        ING_ALLOC(g.coff, kArCoff, nc + 1);
         ING_TRY(cudaMemcpyAsync(g.coff, coff.data(), sizeof(int32_t) * (nc + 1), cudaMemcpyHostToDevice, st));
         ING_TRY(cudaMemcpyAsync(g.cverts, cv.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice, st));
         ING_TRY(cudaStreamSynchronize(st));
@@ -391,9 +396,7 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
     g.slots = slots;
 done:
 #undef ING_TRY
-    cudaFree(d_rp64); cudaFree(d_col); cudaFree(d_sign); cudaFree(d_err);
-    cudaFree(uptr); cudaFree(upc); cudaFree(ebase); cudaFree(tmp); cudaFree(lab);
-    cudaFree(flag); cudaFree(rank);
+#undef ING_ALLOC
     return rc;
 }
 

@@ -163,6 +163,19 @@ void set_error(const std::string &msg);
     } while (0)
 
 // ---------------------------------------------------------------------------
+// Persistent grow-only device buffers for the graph and the ingest
+// temporaries: a reload of a graph that fits reuses them (no cudaMalloc /
+// cudaFree per load; all dynamic memory allocated once, L236).
+// ---------------------------------------------------------------------------
+enum ArenaSlot {
+    kArRowPtr64, kArCol, kArSign, kArErr, kArRowPtr, kArAdj, kArAdjEid, kArEdges, kArComp,
+    kArCverts, kArUptr, kArUpc, kArEbase, kArScanTmp, kArLab, kArFlag, kArRank, kArCoff,
+    kArSlots
+};
+void *arena(int slot, size_t bytes);   // nullptr on allocation failure (error set)
+void arena_free_all();
+
+// ---------------------------------------------------------------------------
 // Launch helpers implemented in the .cu files
 // ---------------------------------------------------------------------------
 int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr,
