@@ -45,6 +45,7 @@ def parse():
     ap.add_argument("--trees", type=int, default=0, help="trees per GPU per step (0 = config default)")
     ap.add_argument("--walk", type=int, default=0)
     ap.add_argument("--batch", type=int, default=0)
+    ap.add_argument("--sub", type=int, default=0, help="trees per labelling launch (0 = auto)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample-trees", type=int, default=0)
@@ -217,6 +218,7 @@ def main():
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     graphb.set_option("walk", args.walk)
     graphb.set_option("batch", args.batch)
+    graphb.set_option("sub", args.sub)
     graphb.load_graph(g)
     n, m, ncomp = graphb.graph_info()
     c_nt = m - n + ncomp

@@ -97,7 +97,8 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
 /* Options (before gb_balance*): "batch" trees per batch (0 = auto),
  * "cycle_group" trees per cycle-kernel pass (0 = auto), "walk"
  * (0 = two-ended interval walk, 1 = Alg. 3 descent with warp ballots),
- * "timing" (1 = record per-phase CUDA events), "graphs" (1 = CUDA graphs). */
+ * "timing" (1 = record per-phase CUDA events), "graphs" (1 = CUDA graphs),
+ * "sub" (trees per labelling launch, 0 = auto), "msprof" (see gb_msbfs_profile). */
 int gb_set_option(const char *key, int64_t value);
 
 /* Statistics of the last gb_balance / gb_balance_range call:
@@ -122,6 +123,13 @@ int gb_get_stats(int64_t *ints, int n_ints, double *phase_ms, int n_phase);
  * 2^-64 collisions -- frustration-cloud analytics, Fig. 2 L81/L86);
  * tree_ids[i] = t.  Returns the count. */
 int64_t gb_tree_stats(uint64_t *out, int64_t *tree_ids, int64_t max_trees);
+
+/* Profiling aid: with option "msprof" = 1, the multi-source BFS of the last
+ * batch records %globaltimer (ns) at its phase boundaries, out[4*L + k] for
+ * level L < 256: k = 0 level start, 1 end of the discovery pass, 2 end of the
+ * parent pass, 3 end of the hub pass (0 = not reached).  out has 1024 entries.
+ * GB_ESTATE if the option is not set. */
+int gb_msbfs_profile(uint64_t *out);
 
 /* Ingest results (§8 a.1), copied to host arrays (any pointer may be NULL):
  * edge_u[m], edge_v[m] (u < v), edge_neg[m] (1 = negative) indexed by eid;

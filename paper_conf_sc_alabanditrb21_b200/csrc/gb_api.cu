@@ -50,6 +50,8 @@ struct Options {
     int64_t cycle_group = 0; // 0 = auto
     int64_t walk = 0;        // 0 two-ended, 1 Alg. 3 descent
     int64_t timing = 0;
+    int64_t sub = 0;         // trees per labelling launch (0 = auto)
+    int64_t msprof = 0;      // record BFS phase timestamps (gb_msbfs_profile)
 };
 
 struct Stats {
@@ -83,7 +85,7 @@ static void free_ws(Workspace &w) {
     void *ptrs[] = {w.vst, w.qv, w.qs, w.qr, w.pkeyq, w.lvl, w.vbase, w.size, w.sz64,
                     w.parq, w.offq, w.szq, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
-                    w.scan_tmp};
+                    w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof};
     for (void *p : ptrs) if (p) cudaFree(p);
     w = Workspace();
 }
@@ -94,7 +96,7 @@ static void free_graph(Graph &g) {
 
 static size_t per_tree_bytes(const Graph &g, bool descent) {
     const size_t n = (size_t)g.n;
-    size_t b = 61 * n + 32 + 4 * (size_t)((g.m + 31) / 32) + 4 * (size_t)g.ncomp;
+    size_t b = 44 * n + 32 + 4 * (size_t)((g.m + 31) / 32) + 4 * (size_t)g.ncomp;
     if (descent) b += 24 * n;
     return b;
 }
@@ -117,11 +119,20 @@ static int ensure_workspace(int B, bool descent) {
     const Graph &g = S.g;
     const int64_t n = g.n, Bn = (int64_t)B * n, words = (g.m + 31) / 32;
     const int64_t nw = (n + 3) / 4;
-    ALLOC(w.vst, (int64_t)B * nw);
+    // push BFS state, used for caller-given trees only (one tree at a time)
+    ALLOC(w.vst, nw);
+    ALLOC(w.qs, n);
+    ALLOC(w.qr, n);
+    ALLOC(w.pkeyq, n);
+    // multi-source BFS state (one bit per tree)
+    ALLOC(w.vis, n);
+    ALLOC(w.fr, 2 * n);
+    ALLOC(w.hacc, std::max<int64_t>(g.nmulti, 1));
+    ALLOC(w.hbest, std::max<int64_t>(g.nmulti, 1) * kMsBatch);
+    ALLOC(w.msflag, 2);
+    ALLOC(w.mscnt, (int64_t)kMsBatch * 2048);
+    ALLOC(w.fbm, 4 * ((n + 31) / 32));
     ALLOC(w.qv, Bn);
-    ALLOC(w.qs, Bn);
-    ALLOC(w.qr, Bn);
-    ALLOC(w.pkeyq, Bn);
     ALLOC(w.lvl, (int64_t)B * (n + 2));
     ALLOC(w.vbase, (int64_t)B * (n + 2));
     ALLOC(w.parq, Bn);
@@ -191,10 +202,16 @@ static int auto_batch(int64_t ntrees) {
     if (S.opt.batch > 0) return (int)std::min<int64_t>(S.opt.batch, kMaxBatch);
     const size_t have = S.free_at_load;
     int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk == 1));
-    int64_t b = std::min<int64_t>({ntrees, (int64_t)kMaxBatch, std::max<int64_t>(bm, 1)});
-    // large graphs: a few trees per batch already fill the GPU
-    if (S.g.n >= (1 << 22)) b = std::min<int64_t>(b, 2);
+    int64_t b = std::min<int64_t>({ntrees, (int64_t)kMsBatch, std::max<int64_t>(bm, 1)});
     return (int)std::max<int64_t>(b, 1);
+}
+
+// trees per labelling launch: large graphs keep one or two trees' random-access
+// arrays (40-80 MB each) L2-resident; small graphs label the whole batch
+static int auto_sub(int B) {
+    if (S.opt.sub > 0) return (int)std::min<int64_t>(S.opt.sub, B);
+    if (S.g.n >= (1 << 22)) return std::min(B, 2);
+    return B;
 }
 
 static int auto_group(int B) {
@@ -219,6 +236,9 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     int rc = ensure_workspace(B, descent);
     if (rc) return rc;
     const int G = auto_group(B);
+    if (S.opt.msprof && !S.ws.msprof) GB_CUDA_TRY(cudaMalloc(&S.ws.msprof, sizeof(unsigned long long) * 1024));
+    if (!S.opt.msprof && S.ws.msprof) { cudaFree(S.ws.msprof); S.ws.msprof = nullptr; }
+    if (S.ws.msprof) GB_CUDA_TRY(cudaMemsetAsync(S.ws.msprof, 0, sizeof(unsigned long long) * 1024, st));
     T.batch_used = B;
     T.group_used = G;
     if (!S.d_rec_stats) {
@@ -240,7 +260,9 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, nb, seed, t0, stride);
         ++T.launches;
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 3 * nb, st));
-        rc = run_batch_tree(S.g, S.ws, nb, nullptr, st, &T.launches, ev, descent);
+        GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
+        GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
+        rc = run_batch_tree(S.g, S.ws, nb, nullptr, st, &T.launches, ev, descent, auto_sub(nb));
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
         rc = run_batch_cycles(S.g, S.ws, nb, G, descent, st, &T.launches);
@@ -291,7 +313,9 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
     k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, 1, seed, t, 1);
     ++T.launches;
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 3, st));
-    rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk == 1);
+    GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
+    GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
+    rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk == 1, 1);
     if (rc) return rc;
     if (d_given) {
         unsigned long long vis = 0;
@@ -389,7 +413,7 @@ int gb_load_csr(int64_t n, int64_t m, const int64_t *row_ptr, const int32_t *col
     // a reload on the same device keeps the tree workspace if the new graph
     // has the same shape (all dynamic memory allocated once, L236)
     const bool same_dev = S.stream != nullptr && S.g.dev == dev;
-    const int64_t old_n = S.g.n, old_m = S.g.m, old_c = S.g.ncomp;
+    const int64_t old_n = S.g.n, old_m = S.g.m, old_c = S.g.ncomp, old_h = S.g.nmulti;
     if (same_dev) release_graph(true); else gb_free();
     int coop = 0;
     GB_CUDA_TRY(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev));
@@ -400,7 +424,8 @@ int gb_load_csr(int64_t n, int64_t m, const int64_t *row_ptr, const int32_t *col
     int64_t launches = 0;
     rc = ingest(S.g, n, m, row_ptr, col_idx, sign, S.stream, &launches);
     if (rc) { gb_free(); return rc; }
-    if (S.ws.B && (S.g.n != old_n || S.g.m != old_m || S.g.ncomp != old_c)) free_ws(S.ws);
+    if (S.ws.B && (S.g.n != old_n || S.g.m != old_m || S.g.ncomp != old_c || S.g.nmulti != old_h))
+        free_ws(S.ws);
     S.h_comp.resize(n);
     GB_CUDA_TRY(cudaMemcpy(S.h_comp.data(), S.g.comp, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
     {
@@ -447,6 +472,8 @@ int gb_set_option(const char *key, int64_t value) {
     else if (!strcmp(key, "cycle_group")) { if (value < 0) return GB_EINVAL; S.opt.cycle_group = value; }
     else if (!strcmp(key, "walk")) { if (value != 0 && value != 1) return GB_EINVAL; S.opt.walk = value; }
     else if (!strcmp(key, "timing")) S.opt.timing = value != 0;
+    else if (!strcmp(key, "sub")) { if (value < 0) return GB_EINVAL; S.opt.sub = value; }
+    else if (!strcmp(key, "msprof")) S.opt.msprof = value != 0;
     else if (!strcmp(key, "graphs")) { /* reserved */ }
     else { set_error(std::string("unknown option ") + key); return GB_EINVAL; }
     return GB_OK;
@@ -544,6 +571,13 @@ int gb_get_stats(int64_t *ints, int n_ints, double *phase_ms, int n_phase) {
     for (; ints && k < n_ints && k < 8; k++) ints[k] = v[k];
     for (int i = 0; phase_ms && i < n_phase && i < GB_NPHASE; i++) phase_ms[i] = T.phase_ms[i];
     return k;
+}
+
+// BFS phase timestamps of the last batch (option "msprof"): [256][4] ns
+int gb_msbfs_profile(uint64_t *out) {
+    if (!S.ws.msprof) { set_error("msprof option not set"); return GB_ESTATE; }
+    GB_CUDA_TRY(cudaMemcpy(out, S.ws.msprof, sizeof(uint64_t) * 1024, cudaMemcpyDeviceToHost));
+    return GB_OK;
 }
 
 int64_t gb_tree_stats(uint64_t *out, int64_t *tree_ids, int64_t max_trees) {

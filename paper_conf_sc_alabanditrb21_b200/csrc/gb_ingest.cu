@@ -13,6 +13,8 @@
 #include "gb_internal.cuh"
 #include "../../include/graphb.h"
 
+#include <cub/device/device_radix_sort.cuh>
+
 #include <algorithm>
 #include <vector>
 
@@ -269,6 +271,43 @@ __global__ void k_cc_rank(const uint32_t *__restrict__ root, const uint32_t *__r
         comp[v] = (int32_t)rank[root[v]];
 }
 
+// ---------------------------------------------------------------------------
+// Degree-sorted view for the multi-source BFS (gb_msbfs.cu)
+// ---------------------------------------------------------------------------
+__global__ void k_degrees(const uint32_t *__restrict__ rp, int64_t n, uint32_t *__restrict__ deg,
+                          uint32_t *__restrict__ ids) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        deg[v] = rp[v + 1] - rp[v];
+        ids[v] = (uint32_t)v;
+    }
+}
+
+__global__ void k_view_rank(const uint32_t *__restrict__ bord, const uint32_t *__restrict__ sdeg,
+                            int64_t n, uint32_t *__restrict__ brank, unsigned long long *counts) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        brank[bord[i]] = (uint32_t)i;
+        const uint32_t d = sdeg[i];
+        if (d > (uint32_t)kLight) atomicAdd(counts, 1ull);
+        if (d > (uint32_t)kChunk) atomicAdd(counts + 1, 1ull);
+    }
+}
+
+__global__ void k_view_slots(const uint32_t *__restrict__ rp, const uint32_t *__restrict__ adj,
+                             const uint32_t *__restrict__ brow, const uint32_t *__restrict__ bord,
+                             const uint32_t *__restrict__ brank, int64_t n, uint64_t slots,
+                             uint32_t *__restrict__ badj, uint32_t *__restrict__ borig) {
+    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < slots;
+         j += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t i = row_of_slot(brow, n, (uint32_t)j);
+        const uint32_t o = bord[i];
+        const uint32_t x = adj[rp[o] + ((uint32_t)j - brow[i])];
+        badj[j] = brank[x & kIdMask] | (x & kNegBit);
+        borig[j] = x & kIdMask;
+    }
+}
+
 static unsigned grid_for(int64_t work, int threads, int sms) {
     int64_t b = (work + threads - 1) / threads;
     int64_t cap = (int64_t)sms * 16;
@@ -389,6 +428,66 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
         ING_ALLOC(g.coff, kArCoff, nc + 1);
         ING_TRY(cudaMemcpyAsync(g.coff, coff.data(), sizeof(int32_t) * (nc + 1), cudaMemcpyHostToDevice, st));
         ING_TRY(cudaMemcpyAsync(g.cverts, cv.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice, st));
+        ING_TRY(cudaStreamSynchronize(st));
+    }
+    {
+        // degree-sorted view: stable radix sort of the degrees (descending),
+        // then the view's CSR with internal neighbour ids and original ids
+        uint32_t *deg = nullptr, *sdeg = nullptr, *ids = nullptr;
+        unsigned long long *cnt2 = nullptr;
+        ING_ALLOC(deg, kArDeg, 3 * n + 8);
+        sdeg = deg + n;
+        ids = deg + 2 * n;
+        cnt2 = (unsigned long long *)(((uintptr_t)(deg + 3 * n) + 7) & ~(uintptr_t)7);
+        ING_ALLOC(g.brow, kArBrow, n + 1);
+        ING_ALLOC(g.bord, kArBord, n);
+        ING_ALLOC(g.brank, kArBrank, n);
+        ING_ALLOC(g.badj, kArBadj, slots);
+        ING_ALLOC(g.borig, kArBorig, slots);
+        k_degrees<<<grid_for(n, 256, sms), 256, 0, st>>>(g.row_ptr, n, deg, ids);
+        ++*launches;
+        size_t sort_bytes = 0;
+        ING_TRY(cub::DeviceRadixSort::SortPairsDescending(nullptr, sort_bytes, deg, sdeg, ids, g.bord,
+                                                          (int)n, 0, 32, st));
+        char *sort_tmp = nullptr;
+        ING_ALLOC(sort_tmp, kArSortTmp, sort_bytes);
+        ING_TRY(cub::DeviceRadixSort::SortPairsDescending(sort_tmp, sort_bytes, deg, sdeg, ids, g.bord,
+                                                          (int)n, 0, 32, st));
+        *launches += 4;
+        ING_TRY(cudaMemsetAsync(cnt2, 0, 2 * sizeof(unsigned long long), st));
+        k_view_rank<<<grid_for(n, 256, sms), 256, 0, st>>>(g.bord, sdeg, n, g.brank, cnt2);
+        ++*launches;
+        rc = exclusive_scan_u32(sdeg, g.brow, n, tmp, ntmp, st, launches);
+        if (rc) goto done;
+        const uint32_t s32 = (uint32_t)slots;
+        ING_TRY(cudaMemcpyAsync(g.brow + n, &s32, sizeof(uint32_t), cudaMemcpyHostToDevice, st));
+        if (slots) {
+            k_view_slots<<<grid_for((int64_t)slots, 256, sms), 256, 0, st>>>(
+                g.row_ptr, g.adj, g.brow, g.bord, g.brank, n, slots, g.badj, g.borig);
+            ++*launches;
+        }
+        unsigned long long hc[2] = {0, 0};
+        ING_TRY(cudaMemcpyAsync(hc, cnt2, sizeof(hc), cudaMemcpyDeviceToHost, st));
+        ING_TRY(cudaStreamSynchronize(st));
+        g.nlight0 = (int64_t)hc[0];
+        g.nmulti = (int64_t)hc[1];
+        // work items: chunks of <= kChunk slots of every vertex heavier than kLight
+        std::vector<uint32_t> hrow((size_t)g.nlight0 + 1);
+        ING_TRY(cudaMemcpyAsync(hrow.data(), g.brow, sizeof(uint32_t) * (g.nlight0 + 1),
+                                cudaMemcpyDeviceToHost, st));
+        ING_TRY(cudaStreamSynchronize(st));
+        std::vector<uint2> it;
+        it.reserve((size_t)g.nlight0 + 16);
+        for (int64_t i = 0; i < g.nlight0; i++) {
+            if (i == g.nmulti) g.nmulti_items = (int64_t)it.size();
+            for (uint32_t s0 = hrow[i]; s0 < hrow[i + 1]; s0 += (uint32_t)kChunk)
+                it.push_back(make_uint2((uint32_t)i, s0));
+        }
+        if (g.nmulti == g.nlight0) g.nmulti_items = (int64_t)it.size();
+        g.nitems = (int64_t)it.size();
+        ING_ALLOC(g.items, kArItems, g.nitems);
+        if (g.nitems)
+            ING_TRY(cudaMemcpyAsync(g.items, it.data(), sizeof(uint2) * g.nitems, cudaMemcpyHostToDevice, st));
         ING_TRY(cudaStreamSynchronize(st));
     }
     g.n = n;

@@ -15,6 +15,9 @@ constexpr int32_t kInf = 0x7F7F7F7F;         // "unvisited" BFS distance (memset
 constexpr uint32_t kNone = 0xFFFFFFFFu;
 constexpr int kMaxBatch = 128;               // trees per batch (smem tables)
 constexpr int kBlock = 256;                  // threads per CTA of the cooperative kernels
+constexpr int kMsBatch = 64;                 // trees per multi-source BFS (one bit each)
+constexpr int kLight = 8;                    // BFS: degree <= kLight -> one lane per vertex
+constexpr int kChunk = 2048;                 // BFS: slots per warp work item of a heavier vertex
 
 // ---------------------------------------------------------------------------
 // Counter-based hash: SplitMix64 finaliser and its inverse (R4).
@@ -51,6 +54,17 @@ __host__ __device__ __forceinline__ uint64_t edge_key(uint64_t tkey, uint32_t e)
 }
 __host__ __device__ __forceinline__ uint32_t edge_of_key(uint64_t tkey, uint64_t key) {
     return (uint32_t)((unmix64(key) - tkey) * kGoldenInv - 1);
+}
+
+// parent key of candidate u for w (reading R4): score in the high word, then
+// (u << 1 | neg): the minimum picks the lowest score, ties to the smaller u,
+// and carries the winner's id and the sign of the tree edge.  score = high
+// 32 bits of mix64(tkey + G * (min(u,w) << 32 | max(u,w))), original ids.
+__device__ __forceinline__ unsigned long long parent_key(uint64_t tk, uint32_t u, uint32_t w,
+                                                         uint32_t neg) {
+    const uint64_t lo = min(u, w), hi = max(u, w);
+    const uint32_t score = (uint32_t)(mix64(tk + kGolden * ((lo << 32) | hi)) >> 32);
+    return ((unsigned long long)score << 32) | ((unsigned long long)u << 1) | neg;
 }
 
 // ---------------------------------------------------------------------------
@@ -102,6 +116,22 @@ struct Graph {
     int32_t *coff = nullptr;            // [ncomp+1] component offsets (pre of the root)
     int32_t *cverts = nullptr;          // [n] vertices grouped by component, ascending
     int32_t cbig = 0;                   // largest component
+    // Degree-sorted view for the multi-source BFS (gb_msbfs.cu): internal ids
+    // 0..n-1 order the vertices by degree, descending (ties by original id),
+    // so a warp's 32 consecutive vertices have similar degrees and the hubs
+    // sit at the front.  Only the BFS uses internal ids; everything it emits
+    // (level lists, parents) is in original ids.
+    uint32_t *brow = nullptr;           // [n+1] row pointers of the view
+    uint32_t *badj = nullptr;           // [2m] internal neighbour id | neg<<31
+    uint32_t *borig = nullptr;          // [2m] original neighbour id
+    uint32_t *bord = nullptr;           // [n] internal -> original
+    uint32_t *brank = nullptr;          // [n] original -> internal
+    uint2 *items = nullptr;             // [nitems] {internal vertex, first slot}: chunks of <= kChunk
+                                        // slots of the vertices with degree > kLight
+    int64_t nlight0 = 0;                // first internal id with degree <= kLight
+    int64_t nitems = 0;
+    int64_t nmulti = 0;                 // vertices with degree > kChunk (internal ids [0, nmulti))
+    int64_t nmulti_items = 0;           // their chunks (items [0, nmulti_items))
     int dev = 0;
     int num_sms = 148;
 };
@@ -126,6 +156,15 @@ struct Workspace {
     uint32_t *pp = nullptr;    // v: pre | pi<<31  (pi = root-path parity)
     uint2 *rec = nullptr;      // pre: {up pre | neg<<31, size}
     uint32_t *fbits = nullptr; // [B][ceil(m/32)] flip bitmask
+    // multi-source BFS state (one bit per tree of the batch, internal ids)
+    unsigned long long *vis = nullptr;  // [n] trees that reached the vertex
+    unsigned long long *fr = nullptr;   // [2][n] frontier of level L / L+1
+    unsigned long long *hacc = nullptr; // [nmulti] discoveries of multi-chunk vertices
+    unsigned long long *hbest = nullptr;// [nmulti][64] their best parent keys
+    int32_t *msflag = nullptr;          // [2] a multi-chunk vertex discovered something
+    uint32_t *mscnt = nullptr;          // [64][2048] per-block discovery counts
+    unsigned long long *msprof = nullptr;  // [256][4] BFS phase timestamps (option "msprof")
+    uint32_t *fbm = nullptr;            // [4][ceil(n/32)] frontier bitmaps (3) + finished bitmap
     uint32_t *s1 = nullptr;    // [B][ncomp] #vertices with pi = 1 per component
     uint64_t *tkey = nullptr;  // [kMaxBatch]
     int32_t *depth = nullptr;  // [kMaxBatch]
@@ -170,6 +209,7 @@ void set_error(const std::string &msg);
 enum ArenaSlot {
     kArRowPtr64, kArCol, kArSign, kArErr, kArRowPtr, kArAdj, kArAdjEid, kArEdges, kArComp,
     kArCverts, kArUptr, kArUpc, kArEbase, kArScanTmp, kArLab, kArFlag, kArRank, kArCoff,
+    kArBrow, kArBadj, kArBorig, kArBord, kArBrank, kArItems, kArDeg, kArSortTmp,
     kArSlots
 };
 void *arena(int slot, size_t bytes);   // nullptr on allocation failure (error set)
@@ -183,7 +223,20 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr,
            int64_t *launches);
 
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
-                   cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent);
+                   cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub);
+
+// multi-source BFS of the B <= kMsBatch sampled trees of a batch (roots, BFS
+// levels, min-hash parents); fills the level lists qv / parq, lvl, vbase, depth
+struct MsBfsOut {
+    uint32_t *qv, *parq, *pp;
+    uint2 *rec, *crec;
+    uint64_t *lvl;
+    uint32_t *vbase;
+    int32_t *depth, *maxd;
+    const uint64_t *tkey;
+};
+int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStream_t st,
+              int64_t *launches);
 
 int debug_tree_views(const Graph &g, Workspace &ws, bool descent, int32_t *d_parent,
                      int32_t *d_dist, int32_t *d_size, cudaStream_t st);

@@ -1,0 +1,677 @@
+// gb_msbfs.cu -- §8 rows a.2 + a.3 for a batch of B <= 64 sampled trees at
+// once: hashed roots, level-synchronous BFS and min-hash parent selection.
+//
+// The paper builds one BFS tree at a time (§3.1, Fig. 11 "spanning tree"
+// 6 %) and rejects one-tree-per-thread for memory and locality on a 12 GB
+// Titan V (L250).  Here the B trees of a batch share every pass over the
+// graph (§8 a.9, multi-source BFS): each vertex carries a 64-bit word with
+// one bit per tree --
+//   vis[v]  trees that have reached v,
+//   F_L[v]  trees in which v is on level L (the frontier),
+// plus two bitmaps with one bit per vertex: "F_L[v] != 0" (the frontier
+// bitmap, 1.25 MB for 10 M vertices: L2-resident, it gates every frontier
+// word gather) and "vis[v] == all trees" (finished vertices are skipped
+// without touching their words).
+//
+// Level L -> L+1 is a *pull* over the unfinished vertices:
+//   new(w) = OR_{u in N(w), F_L[u] != 0} F_L[u]  AND NOT vis(w),
+// one read of w's adjacency serving all B trees.  For every tree t in new(w)
+// the parent of w is the neighbour u with bit t in F_L[u] (one level up)
+// minimising parent_key(t, u, w) (reading R4).  Discoveries go to the
+// per-tree level lists (qv, parq: original ids, the layout the labelling
+// passes stream).
+//
+// Work mapping (degree-sorted internal ids, gb_ingest.cu):
+//   light vertices (degree <= kLight): one lane per vertex;
+//   heavier vertices: warp work items of <= kChunk slots, lanes stride the
+//     slots, lane l keeps the best key of trees l and l+32;
+//   multi-chunk vertices (degree > kChunk, the hubs of Table 1's max degree
+//     column): partial ORs and partial minima of all their chunks are merged
+//     with global atomics (phase C, only when one of them discovered
+//     something on this level).
+#include "gb_internal.cuh"
+#include "../../include/graphb.h"
+
+#include <algorithm>
+
+namespace gb {
+namespace cg = cooperative_groups;
+
+constexpr int kMsMaxBlocks = 2048;   // capacity of the per-block count table
+
+struct MsParams {
+    const uint32_t *brow, *badj, *borig, *bord, *brank;
+    const uint2 *items;
+    const int32_t *coff, *cverts;
+    int64_t n, ncomp, nitems, nmulti_items, nlight0, nmulti, ls, nwords, itemwords;
+    int B;
+    unsigned long long full;
+    unsigned long long *vis, *fr, *hacc, *hbest;
+    uint32_t *fbm;     // [3][nwords] frontier bitmaps (level L % 3)
+    uint32_t *fullbm;  // [nwords] finished vertices
+    int32_t *flag;
+    uint32_t *mscnt;   // [64][kMsMaxBlocks] discoveries per tree per block (phase A)
+    const uint64_t *tkey;
+    uint32_t *qv, *parq, *pp;
+    uint2 *rec, *crec;
+    uint64_t *lvl;
+    uint32_t *vbase;
+    int32_t *depth, *maxd;
+    unsigned long long *prof;   // optional: globaltimer at phase boundaries (block 0)
+};
+
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+#define MS_PROF(slot)                                                        \
+    do {                                                                     \
+        if (P.prof && blockIdx.x == 0 && tid == 0 && L < 256)                \
+            P.prof[(size_t)L * 4 + (slot)] = gtimer();                       \
+    } while (0)
+
+constexpr int kMsWarps = kBlock / 32;
+
+__device__ __forceinline__ uint32_t warp_incl_scan32(uint32_t v) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+        const uint32_t y = __shfl_up_sync(0xFFFFFFFFu, v, d);
+        if (lane >= d) v += y;
+    }
+    return v;
+}
+
+__device__ __forceinline__ unsigned long long warp_or64(unsigned long long v) {
+#pragma unroll
+    for (int d = 16; d; d >>= 1) v |= __shfl_xor_sync(0xFFFFFFFFu, v, d);
+    return v;
+}
+
+__device__ __forceinline__ bool bm_test(const uint32_t *bm, uint32_t u) {
+    return (__ldcg(bm + (u >> 5)) >> (u & 31)) & 1u;
+}
+
+// frontier word of u (0 unless u is on the current level in some tree)
+__device__ __forceinline__ unsigned long long fr_word(const unsigned long long *F, const uint32_t *bm,
+                                                      uint32_t u) {
+    return bm_test(bm, u) ? __ldcg(F + u) : 0ull;
+}
+
+// level-(L+1) entry `pos` of tree t: the vertex and its parent | neg << 31
+__device__ __forceinline__ void ms_emit(const MsParams &P, int t, uint32_t pos, uint32_t ow,
+                                        unsigned long long key) {
+    const size_t o = (size_t)t * P.n + pos;
+    P.qv[o] = ow;
+    P.parq[o] = ((uint32_t)(key >> 1) & kIdMask) | ((uint32_t)key << 31);
+}
+
+__device__ __forceinline__ void ms_emit_par(const MsParams &P, int t, uint32_t pos, uint32_t ow,
+                                            uint32_t par) {
+    const size_t o = (size_t)t * P.n + pos;
+    P.qv[o] = ow;
+    P.parq[o] = par;
+}
+
+// OR of the frontier words over the slots [s0, s1) (one warp, lanes stride)
+__device__ __forceinline__ unsigned long long ms_chunk_or(const MsParams &P, const unsigned long long *F,
+                                                          const uint32_t *bm, uint32_t s0, uint32_t s1) {
+    const int lane = threadIdx.x & 31;
+    unsigned long long acc = 0;
+    uint32_t j = s0 + lane;
+    for (; j + 96 < s1; j += 128) {
+        const uint32_t a0 = __ldg(P.badj + j) & kIdMask, a1 = __ldg(P.badj + j + 32) & kIdMask;
+        const uint32_t a2 = __ldg(P.badj + j + 64) & kIdMask, a3 = __ldg(P.badj + j + 96) & kIdMask;
+        acc |= fr_word(F, bm, a0) | fr_word(F, bm, a1) | fr_word(F, bm, a2) | fr_word(F, bm, a3);
+    }
+    for (; j < s1; j += 32) acc |= fr_word(F, bm, __ldg(P.badj + j) & kIdMask);
+    return warp_or64(acc);
+}
+
+__device__ __forceinline__ unsigned long long warp_min64(unsigned long long v) {
+#pragma unroll
+    for (int d = 16; d; d >>= 1) v = min(v, __shfl_xor_sync(0xFFFFFFFFu, v, d));
+    return v;
+}
+
+// best parent keys of vertex ow over the slots [s0, s1) for the trees in
+// `want` (one warp, lane = slot): per window of 32 slots, for every tree
+// present, the lanes whose neighbour is a candidate hash it and the warp
+// takes the minimum; lane l keeps trees l (b0) and l + 32 (b1).  When the
+// chunk is the whole adjacency and fits one window, a tree with a single
+// candidate takes it without hashing (its key then has score 0, which only
+// matters for the decode).
+__device__ __forceinline__ void ms_chunk_keys(const MsParams &P, const unsigned long long *F,
+                                              const uint32_t *bm, uint32_t s0, uint32_t s1,
+                                              unsigned long long want, uint32_t ow, const uint64_t *s_tk,
+                                              bool whole, unsigned long long &b0, unsigned long long &b1) {
+    const int lane = threadIdx.x & 31;
+    b0 = ~0ull;
+    b1 = ~0ull;
+    const bool one = whole && s1 - s0 <= 32;
+    for (uint32_t base = s0; base < s1; base += 32) {
+        const uint32_t j = base + lane;
+        uint32_t o = 0;
+        unsigned long long f = 0;
+        if (j < s1) {
+            const uint32_t a = __ldg(P.badj + j);
+            f = fr_word(F, bm, a & kIdMask) & want;
+            if (f) o = __ldg(P.borig + j) | (a & kNegBit);
+        }
+        for (unsigned long long rem = warp_or64(f); rem; rem &= rem - 1) {
+            const int t = __ffsll((long long)rem) - 1;
+            const bool has = (f >> t) & 1ull;
+            const uint32_t bal = __ballot_sync(0xFFFFFFFFu, has);
+            unsigned long long key;
+            if (one && !(bal & (bal - 1))) {
+                const uint32_t par = __shfl_sync(0xFFFFFFFFu, o, __ffs(bal) - 1);
+                key = ((unsigned long long)(par & kIdMask) << 1) | (par >> 31);
+            } else {
+                key = has ? parent_key(s_tk[t], o & kIdMask, ow, o >> 31) : ~0ull;
+                key = warp_min64(key);
+            }
+            if (lane == (t & 31)) {
+                if (t < 32) b0 = min(b0, key);
+                else b1 = min(b1, key);
+            }
+        }
+    }
+}
+
+// per-warp scratch of the parent pass (dynamic shared memory)
+struct WarpScratch {
+    uint16_t pl[32 * kMsBatch];          // (lane << 6 | tree) pairs
+    uint32_t km[kMsBatch / 4][32];       // candidate-slot masks: byte (t & 3) of km[t >> 2][lane]
+    uint32_t lo[kLight][32];             // candidate neighbour (original id) | neg << 31
+    uint32_t ow[32];                     // original id of each lane's vertex
+    unsigned long long best[kMsBatch];   // item parents: best key per tree
+};
+constexpr size_t kMsSmem = sizeof(WarpScratch) * kMsWarps;
+
+__device__ __forceinline__ uint32_t key_to_par(unsigned long long key) {
+    return ((uint32_t)(key >> 1) & kIdMask) | ((uint32_t)key << 31);
+}
+
+// parents of the light vertices queued by a warp (lane l: internal id i,
+// valid if `act`) in the trees each discovered on this level (F_{L+1}[i]).
+// Every lane records, per tree, which of its <= kLight neighbours are
+// candidates (one level up in that tree); the (vertex, tree) pairs are then
+// listed and processed one per lane: a single candidate is the parent
+// directly, several go through the min-hash rule (reading R4).
+__device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsigned long long *F,
+                                                 const unsigned long long *Nx, const uint32_t *bm,
+                                                 uint32_t i, bool act, const uint64_t *s_tk,
+                                                 const uint32_t *s_base, uint32_t *s_pos, WarpScratch &W) {
+    const int lane = threadIdx.x & 31;
+    unsigned long long nw = 0;
+#pragma unroll
+    for (int w = 0; w < kMsBatch / 4; w++) W.km[w][lane] = 0;
+    if (act) {
+        nw = __ldcg(Nx + i);
+        const uint32_t rs = __ldg(P.brow + i);
+        const uint32_t deg = __ldg(P.brow + i + 1) - rs;
+        W.ow[lane] = __ldg(P.bord + i);
+#pragma unroll
+        for (int k = 0; k < kLight; k++) {
+            if (k < (int)deg) {
+                const uint32_t a = __ldg(P.badj + rs + k);
+                const unsigned long long c = fr_word(F, bm, a & kIdMask) & nw;
+                if (c) W.lo[k][lane] = __ldg(P.borig + rs + k) | (a & kNegBit);
+                for (unsigned long long m = c; m; m &= m - 1) {
+                    const int t = __ffsll((long long)m) - 1;
+                    W.km[t >> 2][lane] |= (1u << k) << ((t & 3) * 8);
+                }
+            }
+        }
+    }
+    const uint32_t cnt = (uint32_t)__popcll(nw);
+    const uint32_t incl = warp_incl_scan32(cnt);
+    const uint32_t total = __shfl_sync(0xFFFFFFFFu, incl, 31);
+    uint32_t off = incl - cnt;
+    for (unsigned long long m = nw; m; m &= m - 1) W.pl[off++] = (uint16_t)((lane << 6) | (__ffsll((long long)m) - 1));
+    __syncwarp();
+    for (uint32_t p = lane; p < total; p += 32) {
+        const uint32_t e = W.pl[p];
+        const uint32_t src = e >> 6;
+        const int t = (int)(e & 63);
+        uint32_t km = (W.km[t >> 2][src] >> ((t & 3) * 8)) & 0xFFu;
+        const uint32_t ow = W.ow[src];
+        uint32_t par;
+        if (!(km & (km - 1))) {
+            par = W.lo[__ffs(km) - 1][src];   // a single candidate needs no hash
+        } else {
+            const uint64_t tk = s_tk[t];
+            unsigned long long best = ~0ull;
+            for (; km; km &= km - 1) {
+                const uint32_t o = W.lo[__ffs(km) - 1][src];
+                best = min(best, parent_key(tk, o & kIdMask, ow, o >> 31));
+            }
+            par = key_to_par(best);
+        }
+        ms_emit_par(P, t, s_base[t] + atomicAdd(&s_pos[t], 1u), ow, par);
+    }
+    __syncwarp();
+}
+
+// parents of an item vertex whose whole adjacency fits one window (degree
+// <= 32; lane = slot) in the trees `want`: trees with one candidate take it,
+// the (slot, tree) pairs of the others are hashed one per lane and reduced
+// with shared-memory atomicMin.  Lanes l, l + 32 get trees l, l + 32.
+__device__ __forceinline__ void ms_item_parents(const MsParams &P, const unsigned long long *F,
+                                                const uint32_t *bm, uint32_t s0, uint32_t s1,
+                                                unsigned long long want, uint32_t ow,
+                                                const uint64_t *s_tk, WarpScratch &W,
+                                                uint32_t &p0, uint32_t &p1) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t j = s0 + lane;
+    unsigned long long f = 0;
+    uint32_t o = 0;
+    if (j < s1) {
+        const uint32_t a = __ldg(P.badj + j);
+        f = fr_word(F, bm, a & kIdMask) & want;
+        if (f) o = __ldg(P.borig + j) | (a & kNegBit);
+    }
+    unsigned long long s1m = f, s2m = 0;   // trees with >= 1 / >= 2 candidates
+#pragma unroll
+    for (int d = 16; d; d >>= 1) {
+        const unsigned long long o1 = __shfl_xor_sync(0xFFFFFFFFu, s1m, d);
+        const unsigned long long o2 = __shfl_xor_sync(0xFFFFFFFFu, s2m, d);
+        s2m |= o2 | (s1m & o1);
+        s1m |= o1;
+    }
+    W.best[lane] = ~0ull;
+    W.best[lane + 32] = ~0ull;
+    W.lo[0][lane] = o;
+    __syncwarp();
+    for (unsigned long long m = f & ~s2m; m; m &= m - 1)
+        W.best[__ffsll((long long)m) - 1] = ((unsigned long long)(o & kIdMask) << 1) | (o >> 31);
+    const unsigned long long mm = f & s2m;
+    const uint32_t cnt = (uint32_t)__popcll(mm);
+    const uint32_t incl = warp_incl_scan32(cnt);
+    const uint32_t total = __shfl_sync(0xFFFFFFFFu, incl, 31);
+    uint32_t off = incl - cnt;
+    for (unsigned long long m = mm; m; m &= m - 1) W.pl[off++] = (uint16_t)((lane << 6) | (__ffsll((long long)m) - 1));
+    __syncwarp();
+    for (uint32_t p = lane; p < total; p += 32) {
+        const uint32_t e = W.pl[p];
+        const int t = (int)(e & 63);
+        const uint32_t oo = W.lo[0][e >> 6];
+        atomicMin(&W.best[t], parent_key(s_tk[t], oo & kIdMask, ow, oo >> 31));
+    }
+    __syncwarp();
+    p0 = key_to_par(W.best[lane]);
+    p1 = key_to_par(W.best[lane + 32]);
+    __syncwarp();
+}
+
+// position (0-based) of the r-th set bit of m
+__device__ __forceinline__ int select_bit64(unsigned long long m, int r) {
+    int pos = 0;
+    uint32_t x = (uint32_t)m;
+    int c = __popc(x);
+    if (r >= c) { r -= c; x = (uint32_t)(m >> 32); pos = 32; }
+    c = __popc(x & 0xFFFFu); if (r >= c) { r -= c; x >>= 16; pos += 16; }
+    c = __popc(x & 0xFFu);   if (r >= c) { r -= c; x >>= 8;  pos += 8; }
+    c = __popc(x & 0xFu);    if (r >= c) { r -= c; x >>= 4;  pos += 4; }
+    c = __popc(x & 0x3u);    if (r >= c) { r -= c; x >>= 2;  pos += 2; }
+    if (r >= (int)(x & 1u)) pos += 1;
+    return pos;
+}
+
+// ---------------------------------------------------------------------------
+// roots (reading R4): root of component C in tree b = C's vertices
+// (ascending)[rkey(b, C) mod |C|]; level 0 of every tree
+// ---------------------------------------------------------------------------
+__global__ void k_ms_roots(MsParams P) {
+    const int64_t total = (int64_t)P.B * P.ncomp;
+    for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
+         x += (int64_t)gridDim.x * blockDim.x) {
+        const int b = (int)(x / P.ncomp);
+        const int64_t C = x - (int64_t)b * P.ncomp;
+        const uint32_t sz = (uint32_t)(P.coff[C + 1] - P.coff[C]);
+        const uint64_t rk = root_key(P.tkey[b], C);
+        const uint32_t r = (uint32_t)P.cverts[P.coff[C] + (int64_t)(rk % sz)];
+        const uint32_t ri = P.brank[r];
+        const unsigned long long bit = 1ull << b;
+        atomicOr(P.vis + ri, bit);
+        const size_t nb = (size_t)b * P.n;
+        if (P.brow[ri + 1] == P.brow[ri]) {
+            // isolated vertex: a one-vertex tree, finished here (pi = 0)
+            const uint32_t pre = (uint32_t)P.coff[C];
+            P.pp[nb + r] = pre;
+            P.rec[nb + pre] = make_uint2(pre, 1u);
+            if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
+            continue;
+        }
+        const unsigned long long old = atomicAdd((unsigned long long *)(P.lvl + b * P.ls), 1ull << 32);
+        const uint32_t pos = (uint32_t)(old >> 32);
+        P.qv[nb + pos] = r;
+        P.parq[nb + pos] = r;
+        atomicOr(P.fr + ri, bit);
+        atomicOr(P.fbm + (ri >> 5), 1u << (ri & 31));
+    }
+}
+
+// ---------------------------------------------------------------------------
+// the BFS: one cooperative kernel.  Per level L:
+//   phase A  every block pulls over its tiles (static: tile k -> block
+//            k mod grid): new(w), vis, F_{L+1}, the bitmaps; per-tree
+//            discovery counts in shared memory, published per block;
+//   -- grid barrier --
+//   phase B  each block's offset in every tree's level-(L+1) list = the
+//            counts of the blocks before it; the same tiles again: the
+//            parents of the discoveries (light vertices: one (vertex, tree)
+//            pair per lane), written to the level lists; hubs' partial minima;
+//   -- grid barrier --
+//   phase C  (only if a hub discovered something) hubs' parents appended,
+//            then one more barrier.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(kBlock, 3) k_msbfs(MsParams P) {
+    cg::grid_group grid = cg::this_grid();
+    __shared__ uint64_t s_tk[kMsBatch];
+    __shared__ uint32_t s_cnt[kMsBatch], s_pos[kMsBatch], s_base[kMsBatch];
+    __shared__ uint32_t s_vbase[kMsBatch], s_vb[kMsBatch];
+    __shared__ int32_t s_depth[kMsBatch];
+    __shared__ int s_more;
+    extern __shared__ __align__(16) unsigned char s_dyn[];
+    WarpScratch &W = reinterpret_cast<WarpScratch *>(s_dyn)[threadIdx.x >> 5];
+    __shared__ uint32_t s_q[kMsWarps][64];           // discovered light vertices (phase B)
+    uint32_t qn = 0;                                  // warp-uniform fill of s_q
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    const int B = P.B;
+    if (tid < kMsBatch) {
+        s_tk[tid] = tid < B ? P.tkey[tid] : 0;
+        s_cnt[tid] = 0;
+        s_pos[tid] = 0;
+        s_base[tid] = 0;
+        s_vbase[tid] = 0;
+        s_depth[tid] = 0;
+    }
+    const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + tid;
+    const int64_t gwarp = gtid >> 5;
+    const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+    const int64_t nwarps = nthr >> 5;
+    const int64_t nit_tiles = (P.nitems + kMsWarps - 1) / kMsWarps;
+    const int64_t l0 = P.nlight0 & ~31ll;   // light tiles start word-aligned
+    const int64_t nl_tiles = (P.n - l0 + kBlock - 1) / kBlock;
+    const int64_t ntiles = nit_tiles + nl_tiles;
+    const unsigned long long full = P.full;
+    const uint32_t nblk = gridDim.x;
+    for (int L = 0;; L++) {
+        const unsigned long long *F = P.fr + (size_t)(L & 1) * P.n;
+        unsigned long long *Nx = P.fr + (size_t)((L + 1) & 1) * P.n;
+        const uint32_t *bm = P.fbm + (size_t)(L % 3) * P.nwords;
+        uint32_t *nbm = P.fbm + (size_t)((L + 1) % 3) * P.nwords;
+        uint32_t *cbm = P.fbm + (size_t)((L + 2) % 3) * P.nwords;   // free: cleared for L+2
+        __syncthreads();
+        if (tid < B) {
+            const uint32_t c = (uint32_t)(__ldcg((const unsigned long long *)(P.lvl + tid * P.ls + L)) >> 32);
+            s_vb[tid] = s_vbase[tid] + c;   // start of level L+1 in tree tid's list
+            if (blockIdx.x == 0) P.vbase[tid * P.ls + L + 1] = s_vb[tid];
+        }
+        // words written with atomics next level (items, the boundary word)
+        for (int64_t w = gtid; w < P.itemwords; w += nthr) cbm[w] = 0;
+        __syncthreads();
+        MS_PROF(0);
+        // ---------------- phase A: discoveries --------------------------------
+        for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+            if (tile < nit_tiles) {
+                const int64_t k = tile * kMsWarps + wid;
+                if (k < P.nitems) {
+                    const uint2 it = __ldg(P.items + k);
+                    const uint32_t i = it.x, s0 = it.y;
+                    if (bm_test(P.fullbm, i)) continue;
+                    const uint32_t s1 = min(s0 + (uint32_t)kChunk, __ldg(P.brow + i + 1));
+                    const bool multi = k < P.nmulti_items;
+                    const unsigned long long vis = __ldcg(P.vis + i);
+                    const unsigned long long part = ms_chunk_or(P, F, bm, s0, s1) & ~vis;
+                    if (multi) {
+                        if (part && lane == 0) {
+                            atomicOr(P.hacc + i, part);
+                            P.flag[L & 1] = 1;
+                        }
+                    } else if (part) {
+                        if (lane == 0) {
+                            Nx[i] = part;
+                            P.vis[i] = vis | part;
+                            atomicOr(nbm + (i >> 5), 1u << (i & 31));
+                            if ((vis | part) == full) atomicOr(P.fullbm + (i >> 5), 1u << (i & 31));
+                        }
+                        if ((part >> lane) & 1ull) atomicAdd(&s_cnt[lane], 1u);
+                        if ((part >> (lane + 32)) & 1ull) atomicAdd(&s_cnt[lane + 32], 1u);
+                    }
+                }
+            } else {
+                const int64_t v0 = l0 + (tile - nit_tiles) * kBlock + wid * 32;   // this warp's word
+                if (v0 >= P.n) continue;
+                const uint32_t i = (uint32_t)(v0 + lane);
+                const bool mine = (int64_t)i < P.n && (int64_t)i >= P.nlight0;
+                const uint32_t fw = __ldcg(P.fullbm + (v0 >> 5));
+                unsigned long long nw = 0;
+                bool nowfull = false;
+                if (mine && !((fw >> lane) & 1u)) {
+                    const unsigned long long vis = __ldcg(P.vis + i);
+                    const uint32_t rs = __ldg(P.brow + i);
+                    const uint32_t deg = __ldg(P.brow + i + 1) - rs;
+                    unsigned long long acc = 0;
+#pragma unroll
+                    for (int k = 0; k < kLight; k++)
+                        if (k < (int)deg) acc |= fr_word(F, bm, __ldg(P.badj + rs + k) & kIdMask);
+                    nw = acc & ~vis;
+                    if (nw) {
+                        P.vis[i] = vis | nw;
+                        Nx[i] = nw;
+                        nowfull = (vis | nw) == full;
+                        for (unsigned long long r = nw; r; r &= r - 1)
+                            atomicAdd(&s_cnt[__ffsll((long long)r) - 1], 1u);
+                    } else {
+                        nowfull = vis == full;
+                    }
+                }
+                const uint32_t fb = __ballot_sync(0xFFFFFFFFu, nw != 0);
+                const uint32_t nf = __ballot_sync(0xFFFFFFFFu, nowfull);
+                if (lane == 0) {
+                    if (v0 >= P.nlight0) {
+                        nbm[v0 >> 5] = fb;
+                        if (nf) P.fullbm[v0 >> 5] = fw | nf;
+                    } else {   // boundary word shared with item vertices
+                        if (fb) atomicOr(nbm + (v0 >> 5), fb);
+                        if (nf) atomicOr(P.fullbm + (v0 >> 5), nf);
+                    }
+                }
+            }
+        }
+        __syncthreads();
+        if (tid < kMsBatch) {
+            P.mscnt[(size_t)tid * kMsMaxBlocks + blockIdx.x] = s_cnt[tid];
+            s_cnt[tid] = 0;
+        }
+        grid.sync();
+        MS_PROF(1);
+        // ---------------- phase B: parents ------------------------------------
+        // this block's offsets: counts of the blocks before it (warp per tree)
+        for (int t = wid; t < B; t += kMsWarps) {
+            const uint32_t *row = P.mscnt + (size_t)t * kMsMaxBlocks;
+            uint32_t before = 0, all = 0;
+            for (uint32_t b = lane; b < nblk; b += 32) {
+                const uint32_t c = __ldcg(row + b);
+                all += c;
+                if (b < blockIdx.x) before += c;
+            }
+#pragma unroll
+            for (int d = 16; d; d >>= 1) {
+                before += __shfl_xor_sync(0xFFFFFFFFu, before, d);
+                all += __shfl_xor_sync(0xFFFFFFFFu, all, d);
+            }
+            if (lane == 0) {
+                s_base[t] = s_vb[t] + before;
+                s_pos[t] = 0;
+                if (blockIdx.x == 0) P.lvl[t * P.ls + L + 1] = (uint64_t)all << 32;
+            }
+        }
+        __syncthreads();
+        for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+            if (tile < nit_tiles) {
+                const int64_t k = tile * kMsWarps + wid;
+                if (k < P.nitems && k >= P.nmulti_items) {
+                    const uint2 it = __ldg(P.items + k);
+                    const uint32_t i = it.x;
+                    if (!bm_test(nbm, i)) continue;
+                    const unsigned long long nw = __ldcg(Nx + i);
+                    const uint32_t s1 = min(it.y + (uint32_t)kChunk, __ldg(P.brow + i + 1));
+                    const uint32_t ow = __ldg(P.bord + i);
+                    uint32_t p0, p1;
+                    if (s1 - it.y <= 32) {
+                        ms_item_parents(P, F, bm, it.y, s1, nw, ow, s_tk, W, p0, p1);
+                    } else {
+                        unsigned long long b0, b1;
+                        ms_chunk_keys(P, F, bm, it.y, s1, nw, ow, s_tk, true, b0, b1);
+                        p0 = key_to_par(b0);
+                        p1 = key_to_par(b1);
+                    }
+                    if ((nw >> lane) & 1ull)
+                        ms_emit_par(P, lane, s_base[lane] + atomicAdd(&s_pos[lane], 1u), ow, p0);
+                    if ((nw >> (lane + 32)) & 1ull)
+                        ms_emit_par(P, lane + 32, s_base[lane + 32] + atomicAdd(&s_pos[lane + 32], 1u), ow, p1);
+                }
+            } else {
+                // light vertices: the warp queues its discovered vertices and
+                // processes them 32 at a time (one per lane)
+                const int64_t v0 = l0 + (tile - nit_tiles) * kBlock + wid * 32;
+                if (v0 >= P.n) continue;
+                uint32_t fb = __ldcg(nbm + (v0 >> 5));
+                if (v0 < P.nlight0) fb &= ~0u << (uint32_t)(P.nlight0 - v0);   // item lanes are not ours
+                if (!fb) continue;
+                if ((fb >> lane) & 1u) s_q[wid][qn + __popc(fb & ((1u << lane) - 1u))] = (uint32_t)(v0 + lane);
+                qn += __popc(fb);
+                if (qn >= 32) {
+                    __syncwarp();
+                    const uint32_t i = s_q[wid][lane];
+                    const uint32_t rest = s_q[wid][32 + lane];
+                    __syncwarp();
+                    s_q[wid][lane] = rest;
+                    qn -= 32;
+                    ms_light_parents(P, F, Nx, bm, i, true, s_tk, s_base, s_pos, W);
+                }
+            }
+        }
+        __syncwarp();
+        if (qn) ms_light_parents(P, F, Nx, bm, s_q[wid][lane], lane < qn, s_tk, s_base, s_pos, W);
+        qn = 0;
+        // hubs: partial minima of every chunk
+        const bool multi = P.nmulti_items > 0 && *(volatile int32_t *)(P.flag + (L & 1)) != 0;
+        if (multi) {
+            for (int64_t k = gwarp; k < P.nmulti_items; k += nwarps) {
+                const uint2 it = __ldg(P.items + k);
+                const uint32_t hi = it.x;
+                const unsigned long long want = __ldcg(P.hacc + hi);
+                if (!want) continue;
+                const uint32_t e1 = min(it.y + (uint32_t)kChunk, __ldg(P.brow + hi + 1));
+                unsigned long long b0, b1;
+                ms_chunk_keys(P, F, bm, it.y, e1, want, __ldg(P.bord + hi), s_tk, false, b0, b1);
+                if (b0 != ~0ull) atomicMin(P.hbest + (size_t)hi * kMsBatch + lane, b0);
+                if (b1 != ~0ull) atomicMin(P.hbest + (size_t)hi * kMsBatch + lane + 32, b1);
+            }
+        }
+        if (blockIdx.x == 0 && tid == 0) P.flag[(L + 1) & 1] = 0;
+        grid.sync();
+        MS_PROF(2);
+        // ---------------- phase C: hubs -----------------------------------------
+        if (multi) {
+            for (int64_t hi = gwarp; hi < P.nmulti; hi += nwarps) {
+                const unsigned long long want = __ldcg(P.hacc + hi);
+                if (!want) continue;
+                const uint32_t ow = __ldg(P.bord + hi);
+#pragma unroll
+                for (int h = 0; h < 2; h++) {
+                    const int t = lane + 32 * h;
+                    if ((want >> t) & 1ull) {
+                        unsigned long long *slot = P.hbest + (size_t)hi * kMsBatch + t;
+                        const unsigned long long key = __ldcg(slot);
+                        *slot = ~0ull;
+                        const unsigned long long old =
+                            atomicAdd((unsigned long long *)(P.lvl + t * P.ls + L + 1), 1ull << 32);
+                        ms_emit(P, t, s_vb[t] + (uint32_t)(old >> 32), ow, key);
+                    }
+                }
+                __syncwarp();
+                if (lane == 0) {
+                    const unsigned long long vis = __ldcg(P.vis + hi) | want;
+                    P.vis[hi] = vis;
+                    Nx[hi] = want;
+                    P.hacc[hi] = 0;
+                    atomicOr(nbm + (hi >> 5), 1u << (hi & 31));
+                    if (vis == full) atomicOr(P.fullbm + (hi >> 5), 1u << (hi & 31));
+                }
+            }
+            grid.sync();
+        }
+        MS_PROF(3);
+        // ---------------- next level or done --------------------------------
+        if (tid == 0) s_more = 0;
+        __syncthreads();
+        if (tid < B) {
+            const uint32_t cc = (uint32_t)(__ldcg((const unsigned long long *)(P.lvl + tid * P.ls + L + 1)) >> 32);
+            if (cc) {
+                s_depth[tid] = L + 1;
+                atomicOr(&s_more, 1);
+            }
+            s_vbase[tid] = s_vb[tid];
+        }
+        __syncthreads();
+        if (!s_more) break;
+    }
+    if (blockIdx.x == 0 && tid < B) {
+        P.depth[tid] = s_depth[tid];
+        atomicMax(P.maxd, s_depth[tid]);
+    }
+}
+
+// ---------------------------------------------------------------------------
+// host side
+// ---------------------------------------------------------------------------
+int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStream_t st,
+              int64_t *launches) {
+    if (B < 1 || B > kMsBatch) { set_error("msbfs: batch out of range"); return GB_EINVAL; }
+    static int blocks = 0;
+    if (!blocks) {
+        int per = 0;
+        GB_CUDA_TRY(cudaFuncSetAttribute(k_msbfs, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMsSmem));
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_msbfs, kBlock, kMsSmem) != cudaSuccess || per < 1)
+            per = 1;
+        blocks = std::min(per * g.num_sms, kMsMaxBlocks);
+    }
+    MsParams P;
+    P.brow = g.brow; P.badj = g.badj; P.borig = g.borig; P.bord = g.bord; P.brank = g.brank;
+    P.items = g.items; P.coff = g.coff; P.cverts = g.cverts;
+    P.n = g.n; P.ncomp = g.ncomp; P.nitems = g.nitems; P.nmulti_items = g.nmulti_items;
+    P.nlight0 = g.nlight0; P.nmulti = g.nmulti; P.ls = g.n + 2;
+    P.nwords = (g.n + 31) / 32;
+    P.itemwords = (g.nlight0 + 31) / 32;
+    P.B = B;
+    P.full = B == 64 ? ~0ull : ((1ull << B) - 1);
+    P.vis = ws.vis; P.fr = ws.fr; P.hacc = ws.hacc; P.hbest = ws.hbest;
+    P.fbm = ws.fbm; P.fullbm = ws.fbm + 3 * P.nwords;
+    P.flag = ws.msflag; P.mscnt = ws.mscnt;
+    P.tkey = o.tkey; P.qv = o.qv; P.parq = o.parq; P.pp = o.pp; P.rec = o.rec; P.crec = o.crec;
+    P.lvl = o.lvl; P.vbase = o.vbase; P.depth = o.depth; P.maxd = o.maxd;
+    P.prof = ws.msprof;
+    GB_CUDA_TRY(cudaMemsetAsync(ws.vis, 0, sizeof(unsigned long long) * (size_t)g.n, st));
+    GB_CUDA_TRY(cudaMemsetAsync(ws.fr, 0, sizeof(unsigned long long) * (size_t)g.n, st));
+    GB_CUDA_TRY(cudaMemsetAsync(ws.fbm, 0, sizeof(uint32_t) * 4 * (size_t)P.nwords, st));
+    GB_CUDA_TRY(cudaMemsetAsync(ws.msflag, 0, sizeof(int32_t) * 2, st));
+    const int64_t work = (int64_t)B * g.ncomp;
+    k_ms_roots<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, 8192)), 256, 0, st>>>(P);
+    ++*launches;
+    void *args[] = {&P};
+    cudaError_t e = cudaLaunchCooperativeKernel((const void *)k_msbfs, dim3(blocks), dim3(kBlock), args, kMsSmem, st);
+    if (e != cudaSuccess) {
+        set_error(std::string("cooperative launch (msbfs): ") + cudaGetErrorString(e));
+        return GB_ECUDA;
+    }
+    ++*launches;
+    return GB_OK;
+}
+
+}  // namespace gb

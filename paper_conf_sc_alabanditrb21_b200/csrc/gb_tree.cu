@@ -78,16 +78,6 @@ __device__ __forceinline__ uint32_t warp_incl_scan32(uint32_t v) {
 // BFS level stamps (see the header comment)
 __device__ __forceinline__ uint32_t level_stamp(int L) { return 0x81u + (uint32_t)(L % 127); }
 
-// parent key of candidate u for w (reading R4): score in the high word, then
-// (u << 1 | neg): the minimum picks the lowest score, ties to the smaller u,
-// and carries the winner's id and the sign of the tree edge
-__device__ __forceinline__ unsigned long long parent_key(uint64_t tk, uint32_t u, uint32_t w,
-                                                         uint32_t neg) {
-    const uint64_t lo = min(u, w), hi = max(u, w);
-    const uint32_t score = (uint32_t)(mix64(tk + kGolden * ((lo << 32) | hi)) >> 32);
-    return ((unsigned long long)score << 32) | ((unsigned long long)u << 1) | neg;
-}
-
 // ---------------------------------------------------------------------------
 // batch reset + roots (a.2)
 // ---------------------------------------------------------------------------
@@ -484,9 +474,9 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
                 nb = (size_t)b * P.n;
                 qi = nb + T.vb[b] + (uint32_t)(i - T.soff[b]);
                 w = __ldcg(P.qv + qi);
-                const uint32_t k = (uint32_t)__ldcg(P.pkeyq + qi);
-                p = k >> 1;
-                neg = k << 31;
+                const uint32_t pq = __ldcg(P.parq + qi);
+                p = pq & kIdMask;
+                neg = pq & kNegBit;
                 // counters hold the sum of the children's sizes: size = 1 + that
                 sz = 1 + (kDescent ? (uint32_t)__ldcg(P.sz64 + nb + w) : __ldcg(P.size + nb + w));
             }
@@ -501,10 +491,7 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
                 const uint32_t o = aggregated_add<uint32_t>(P.size + nb + p, sz, valid);
                 if (valid) P.offq[qi] = 1 + o;
             }
-            if (valid) {
-                P.parq[qi] = p | neg;
-                P.szq[qi] = sz;
-            }
+            if (valid) P.szq[qi] = sz;
         }
         grid.sync();
     }
@@ -632,6 +619,15 @@ __global__ void k_child_counts(TreeParams P, int64_t cnt) {
         P.cstart[i] = (uint32_t)(P.sz64[i] >> 32);
 }
 
+// caller trees (push BFS): parent keys -> parent | neg << 31 in queue order
+__global__ void k_pkey_to_parq(const unsigned long long *pkeyq, uint32_t *parq, int64_t cnt) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cnt;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const unsigned long long k = pkeyq[i];
+        parq[i] = ((uint32_t)(k >> 1) & kIdMask) | ((uint32_t)k << 31);
+    }
+}
+
 // ---------------------------------------------------------------------------
 // debug views of one tree (b = 0): parent / dist / size by vertex
 // ---------------------------------------------------------------------------
@@ -679,8 +675,9 @@ static int launch_coop(const void *fn, int blocks, TreeParams &P, cudaStream_t s
     return GB_OK;
 }
 
+// trees b0 .. b0+B-1 of the workspace
 static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_t *given,
-                              bool descent) {
+                              bool descent, int b0 = 0) {
     TreeParams P;
     P.row_ptr = g.row_ptr; P.adj = g.adj;
     P.comp = g.comp; P.coff = g.coff; P.cverts = g.cverts;
@@ -698,11 +695,24 @@ static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_
     P.clist = descent ? ws.clist : nullptr;
     P.crec = descent ? ws.crec : nullptr;
     P.visited = given ? ws.visited : nullptr;
+    if (b0) {
+        const size_t nb = (size_t)b0 * g.n, lb = (size_t)b0 * P.ls;
+        P.qv += nb; P.parq += nb; P.offq += nb; P.szq += nb; P.pp += nb; P.rec += nb;
+        if (P.size) P.size += nb;
+        if (P.sz64) P.sz64 += nb;
+        if (P.cidxq) P.cidxq += nb;
+        if (P.cstart) P.cstart += nb;
+        if (P.crec) P.crec += nb;
+        P.lvl += lb; P.vbase += lb;
+        P.s1 += (size_t)b0 * g.ncomp;
+        P.tkey += b0; P.depth += b0;
+        P.vst = nullptr; P.qs = nullptr; P.qr = nullptr; P.pkeyq = nullptr;
+    }
     return P;
 }
 
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
-                   cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent) {
+                   cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub) {
     static int bfs_blocks = 0, up_blocks[2] = {0, 0}, down_blocks[2] = {0, 0};
     if (!bfs_blocks) {
         bfs_blocks = coop_blocks((const void *)k_bfs, g.num_sms);
@@ -711,44 +721,61 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
         down_blocks[0] = coop_blocks((const void *)k_top_down<false>, g.num_sms);
         down_blocks[1] = coop_blocks((const void *)k_top_down<true>, g.num_sms);
     }
+    if (sub < 1 || sub > B) sub = B;
     TreeParams P = make_params(g, ws, B, given_parent, descent);
-    const size_t nw = (size_t)P.nw;
     if (ev) GB_CUDA_TRY(cudaEventRecord(ev[0], st));
-    GB_CUDA_TRY(cudaMemsetAsync(ws.vst, 0, sizeof(uint32_t) * (size_t)B * nw, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.s1, 0, sizeof(uint32_t) * (size_t)B * g.ncomp, st));
     if (descent) GB_CUDA_TRY(cudaMemsetAsync(ws.sz64, 0, sizeof(unsigned long long) * (size_t)B * g.n, st));
     else GB_CUDA_TRY(cudaMemsetAsync(ws.size, 0, sizeof(uint32_t) * (size_t)B * g.n, st));
     k_batch_prep<<<1, kMaxBatch, 0, st>>>(P);
     ++*launches;
     if (given_parent) {
+        // a caller tree (B = 1): push BFS along its parent edges
+        GB_CUDA_TRY(cudaMemsetAsync(ws.vst, 0, sizeof(uint32_t) * (size_t)P.nw, st));
         k_roots_given<<<(unsigned)std::min<int64_t>((g.n + 255) / 256, 4096), 256, 0, st>>>(P);
+        ++*launches;
+        GB_CUDA_TRY(cudaGetLastError());
+        if (ev) GB_CUDA_TRY(cudaEventRecord(ev[1], st));
+        int rc = launch_coop((const void *)k_bfs, bfs_blocks, P, st);
+        if (rc) return rc;
+        ++*launches;
+        k_pkey_to_parq<<<(unsigned)std::min<int64_t>((g.n + 255) / 256, 4096), 256, 0, st>>>(ws.pkeyq, ws.parq, g.n);
+        ++*launches;
     } else {
-        const int64_t work = (int64_t)B * g.ncomp;
-        k_roots<<<(unsigned)std::min<int64_t>((work + 255) / 256, 4096), 256, 0, st>>>(P);
+        if (ev) GB_CUDA_TRY(cudaEventRecord(ev[1], st));
+        MsBfsOut o;
+        o.qv = ws.qv; o.parq = ws.parq; o.pp = ws.pp; o.rec = ws.rec;
+        o.crec = descent ? ws.crec : nullptr;
+        o.lvl = ws.lvl; o.vbase = ws.vbase; o.depth = ws.depth; o.maxd = ws.maxd; o.tkey = ws.tkey;
+        int rc = run_msbfs(g, ws, B, o, st, launches);
+        if (rc) return rc;
     }
-    ++*launches;
     GB_CUDA_TRY(cudaGetLastError());
-    if (ev) GB_CUDA_TRY(cudaEventRecord(ev[1], st));
-    int rc = launch_coop((const void *)k_bfs, bfs_blocks, P, st);
-    if (rc) return rc;
-    ++*launches;
     if (ev) GB_CUDA_TRY(cudaEventRecord(ev[2], st));
-    rc = descent ? launch_coop((const void *)k_bottom_up<true>, up_blocks[1], P, st)
-                 : launch_coop((const void *)k_bottom_up<false>, up_blocks[0], P, st);
-    if (rc) return rc;
-    ++*launches;
+    // Alg. 4 on sub-batches of `sub` trees (their random-access arrays stay
+    // L2-resident): all bottom-up passes, then all top-down passes
+    for (int b0 = 0; b0 < B; b0 += sub) {
+        TreeParams Q = make_params(g, ws, std::min(sub, B - b0), given_parent, descent, b0);
+        int rc = descent ? launch_coop((const void *)k_bottom_up<true>, up_blocks[1], Q, st)
+                         : launch_coop((const void *)k_bottom_up<false>, up_blocks[0], Q, st);
+        if (rc) return rc;
+        ++*launches;
+    }
     if (descent) {
         const int64_t cnt = (int64_t)B * g.n;
         k_child_counts<<<(unsigned)std::min<int64_t>((cnt + 255) / 256, 8192), 256, 0, st>>>(P, cnt);
         ++*launches;
-        rc = exclusive_scan_u32(ws.cstart, ws.cstart, cnt, ws.scan_tmp, ws.scan_tmp_elems, st, launches);
+        int rc = exclusive_scan_u32(ws.cstart, ws.cstart, cnt, ws.scan_tmp, ws.scan_tmp_elems, st, launches);
         if (rc) return rc;
     }
     if (ev) GB_CUDA_TRY(cudaEventRecord(ev[3], st));
-    rc = descent ? launch_coop((const void *)k_top_down<true>, down_blocks[1], P, st)
-                 : launch_coop((const void *)k_top_down<false>, down_blocks[0], P, st);
-    if (rc) return rc;
-    ++*launches;
+    for (int b0 = 0; b0 < B; b0 += sub) {
+        TreeParams Q = make_params(g, ws, std::min(sub, B - b0), given_parent, descent, b0);
+        int rc = descent ? launch_coop((const void *)k_top_down<true>, down_blocks[1], Q, st)
+                         : launch_coop((const void *)k_top_down<false>, down_blocks[0], Q, st);
+        if (rc) return rc;
+        ++*launches;
+    }
     return GB_OK;
 }
 

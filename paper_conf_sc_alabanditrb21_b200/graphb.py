@@ -57,6 +57,7 @@ def lib():
         "gb_set_option": (i32, [ctypes.c_char_p, i64]),
         "gb_get_stats": (i32, [P, i32, P, i32]),
         "gb_tree_stats": (i64, [P, P, i64]),
+        "gb_msbfs_profile": (i32, [P]),
         "gb_graph_info": (i32, [P, P, P]),
         "gb_graph_debug": (i32, [P, P, P, P, P]),
         "gb_selftest": (i32, []),
@@ -73,7 +74,7 @@ def lib():
 def exported_symbols():
     return ["gb_load_csr", "gb_balance", "gb_free", "gb_balance_range", "gb_tree_debug",
             "gb_balance_given_tree", "gb_set_option", "gb_get_stats", "gb_tree_stats",
-            "gb_graph_info", "gb_graph_debug", "gb_selftest", "gb_last_error"]
+            "gb_graph_info", "gb_graph_debug", "gb_selftest", "gb_last_error", "gb_msbfs_profile"]
 
 
 def _check(rc):
@@ -255,3 +256,18 @@ def cloud_states(max_trees=1 << 16):
     _, per = tree_stats(max_trees)
     sigs, counts = np.unique(per[:, 3], return_counts=True)
     return {int(s): int(c) for s, c in zip(sigs, counts)}
+
+
+def msbfs_profile():
+    """Per-level BFS phase times (ms) of the last batch: list of
+    (level, discovery, parents, hubs) -- needs set_option("msprof", 1)."""
+    out = np.zeros(1024, dtype=np.uint64)
+    _check(lib().gb_msbfs_profile(_ptr(out)))
+    t = out.reshape(256, 4).astype(np.int64)
+    rows = []
+    for L in range(256):
+        if t[L, 0] == 0:
+            break
+        nxt = t[L + 1, 0] if L + 1 < 256 and t[L + 1, 0] else t[L, 3]
+        rows.append((L, (t[L, 1] - t[L, 0]) / 1e6, (t[L, 2] - t[L, 1]) / 1e6, (nxt - t[L, 2]) / 1e6))
+    return rows
