@@ -17,7 +17,7 @@ constexpr int kMaxBatch = 128;               // trees per batch (smem tables)
 constexpr int kBlock = 256;                  // threads per CTA of the cooperative kernels
 constexpr int kMsBatch = 64;                 // trees per multi-source BFS (one bit each)
 constexpr int kLight = 8;                    // BFS: degree <= kLight -> one lane per vertex
-constexpr int kChunk = 2048;                 // BFS: slots per warp work item of a heavier vertex
+constexpr int kChunk = 256;                  // BFS: slots per warp work item of a heavier vertex
 
 // ---------------------------------------------------------------------------
 // Counter-based hash: SplitMix64 finaliser and its inverse (R4).

@@ -180,9 +180,10 @@ __device__ __forceinline__ void ms_chunk_keys(const MsParams &P, const unsigned 
 }
 
 // per-warp scratch of the parent pass (dynamic shared memory)
+constexpr int kMultiCap = 512;           // multi-candidate pairs per round
 struct WarpScratch {
-    uint16_t pl[32 * kMsBatch];          // (lane << 6 | tree) pairs
-    uint32_t km[kMsBatch / 4][32];       // candidate-slot masks: byte (t & 3) of km[t >> 2][lane]
+    uint32_t ml[kMultiCap];              // multi-candidate pairs: src << 14 | tree << 8 | slot mask
+    uint8_t sidx[kMsBatch][32];          // single-candidate slot of (tree, lane)
     uint32_t lo[kLight][32];             // candidate neighbour (original id) | neg << 31
     uint32_t ow[32];                     // original id of each lane's vertex
     unsigned long long best[kMsBatch];   // item parents: best key per tree
@@ -195,61 +196,90 @@ __device__ __forceinline__ uint32_t key_to_par(unsigned long long key) {
 
 // parents of the light vertices queued by a warp (lane l: internal id i,
 // valid if `act`) in the trees each discovered on this level (F_{L+1}[i]).
-// Every lane records, per tree, which of its <= kLight neighbours are
-// candidates (one level up in that tree); the (vertex, tree) pairs are then
-// listed and processed one per lane: a single candidate is the parent
-// directly, several go through the min-hash rule (reading R4).
+// Trees in which a vertex has a single candidate (one neighbour one level
+// up) take it: the warp walks those trees, the lanes concerned take
+// consecutive positions of the tree's level list (coalesced writes).  The
+// (vertex, tree) pairs with several candidates are listed and hashed one per
+// lane (the min-hash rule, reading R4).
 __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsigned long long *F,
                                                  const unsigned long long *Nx, const uint32_t *bm,
                                                  uint32_t i, bool act, const uint64_t *s_tk,
                                                  const uint32_t *s_base, uint32_t *s_pos, WarpScratch &W) {
     const int lane = threadIdx.x & 31;
-    unsigned long long nw = 0;
-#pragma unroll
-    for (int w = 0; w < kMsBatch / 4; w++) W.km[w][lane] = 0;
+    unsigned long long nw = 0, s2m = 0;   // discovered trees / those with >= 2 candidates
+    unsigned long long c[kLight];
+    uint32_t ow = 0;
     if (act) {
         nw = __ldcg(Nx + i);
         const uint32_t rs = __ldg(P.brow + i);
         const uint32_t deg = __ldg(P.brow + i + 1) - rs;
-        W.ow[lane] = __ldg(P.bord + i);
+        ow = __ldg(P.bord + i);
+        unsigned long long s1m = 0;
 #pragma unroll
         for (int k = 0; k < kLight; k++) {
+            c[k] = 0;
             if (k < (int)deg) {
                 const uint32_t a = __ldg(P.badj + rs + k);
-                const unsigned long long c = fr_word(F, bm, a & kIdMask) & nw;
-                if (c) W.lo[k][lane] = __ldg(P.borig + rs + k) | (a & kNegBit);
-                for (unsigned long long m = c; m; m &= m - 1) {
-                    const int t = __ffsll((long long)m) - 1;
-                    W.km[t >> 2][lane] |= (1u << k) << ((t & 3) * 8);
-                }
+                c[k] = fr_word(F, bm, a & kIdMask) & nw;
+                if (c[k]) W.lo[k][lane] = __ldg(P.borig + rs + k) | (a & kNegBit);
+                s2m |= s1m & c[k];
+                s1m |= c[k];
             }
         }
+#pragma unroll
+        for (int k = 0; k < kLight; k++)
+            for (unsigned long long m = c[k] & ~s2m; m; m &= m - 1) W.sidx[__ffsll((long long)m) - 1][lane] = (uint8_t)k;
+    } else {
+#pragma unroll
+        for (int k = 0; k < kLight; k++) c[k] = 0;
     }
-    const uint32_t cnt = (uint32_t)__popcll(nw);
+    W.ow[lane] = ow;
+    // several candidates: listed pairs, hashed one per lane
+    const uint32_t cnt = (uint32_t)__popcll(s2m);
     const uint32_t incl = warp_incl_scan32(cnt);
     const uint32_t total = __shfl_sync(0xFFFFFFFFu, incl, 31);
-    uint32_t off = incl - cnt;
-    for (unsigned long long m = nw; m; m &= m - 1) W.pl[off++] = (uint16_t)((lane << 6) | (__ffsll((long long)m) - 1));
-    __syncwarp();
-    for (uint32_t p = lane; p < total; p += 32) {
-        const uint32_t e = W.pl[p];
-        const uint32_t src = e >> 6;
-        const int t = (int)(e & 63);
-        uint32_t km = (W.km[t >> 2][src] >> ((t & 3) * 8)) & 0xFFu;
-        const uint32_t ow = W.ow[src];
-        uint32_t par;
-        if (!(km & (km - 1))) {
-            par = W.lo[__ffs(km) - 1][src];   // a single candidate needs no hash
-        } else {
+    for (uint32_t r0 = 0; r0 < total; r0 += kMultiCap) {
+        uint32_t off = incl - cnt;
+        for (unsigned long long m = s2m; m; m &= m - 1) {
+            if (off >= r0 + kMultiCap) break;
+            if (off >= r0) {
+                const int t = __ffsll((long long)m) - 1;
+                uint32_t km = 0;
+#pragma unroll
+                for (int k = 0; k < kLight; k++) km |= (uint32_t)((c[k] >> t) & 1ull) << k;
+                W.ml[off - r0] = ((uint32_t)lane << 14) | ((uint32_t)t << 8) | km;
+            }
+            off++;
+        }
+        __syncwarp();
+        const uint32_t nr = min(total - r0, (uint32_t)kMultiCap);
+        for (uint32_t p = lane; p < nr; p += 32) {
+            const uint32_t e = W.ml[p];
+            const uint32_t src = e >> 14;
+            const int t = (int)((e >> 8) & 63);
+            const uint32_t o_w = W.ow[src];
             const uint64_t tk = s_tk[t];
             unsigned long long best = ~0ull;
-            for (; km; km &= km - 1) {
+            for (uint32_t km = e & 0xFFu; km; km &= km - 1) {
                 const uint32_t o = W.lo[__ffs(km) - 1][src];
-                best = min(best, parent_key(tk, o & kIdMask, ow, o >> 31));
+                best = min(best, parent_key(tk, o & kIdMask, o_w, o >> 31));
             }
-            par = key_to_par(best);
+            ms_emit(P, t, s_base[t] + atomicAdd(&s_pos[t], 1u), o_w, best);
         }
-        ms_emit_par(P, t, s_base[t] + atomicAdd(&s_pos[t], 1u), ow, par);
+        __syncwarp();
+    }
+    // single candidate: no hash; tree by tree, coalesced
+    const unsigned long long sm = nw & ~s2m;
+    const uint32_t lt = (1u << lane) - 1u;
+    for (unsigned long long rem = warp_or64(sm); rem; rem &= rem - 1) {
+        const int t = __ffsll((long long)rem) - 1;
+        const bool has = (sm >> t) & 1ull;
+        const uint32_t mask = __ballot_sync(0xFFFFFFFFu, has);
+        const int leader = __ffs(mask) - 1;
+        uint32_t b = 0;
+        if (lane == leader) b = atomicAdd(&s_pos[t], (uint32_t)__popc(mask));
+        b = __shfl_sync(0xFFFFFFFFu, b, leader);
+        if (has) ms_emit_par(P, t, s_base[t] + b + (uint32_t)__popc(mask & lt), ow, W.lo[W.sidx[t][lane]][lane]);
     }
     __syncwarp();
 }
@@ -264,6 +294,7 @@ __device__ __forceinline__ void ms_item_parents(const MsParams &P, const unsigne
                                                 const uint64_t *s_tk, WarpScratch &W,
                                                 uint32_t &p0, uint32_t &p1) {
     const int lane = threadIdx.x & 31;
+    uint16_t *pl = reinterpret_cast<uint16_t *>(W.ml);   // <= 32 * 64 pairs fit kMultiCap * 2
     const uint32_t j = s0 + lane;
     unsigned long long f = 0;
     uint32_t o = 0;
@@ -290,16 +321,24 @@ __device__ __forceinline__ void ms_item_parents(const MsParams &P, const unsigne
     const uint32_t cnt = (uint32_t)__popcll(mm);
     const uint32_t incl = warp_incl_scan32(cnt);
     const uint32_t total = __shfl_sync(0xFFFFFFFFu, incl, 31);
-    uint32_t off = incl - cnt;
-    for (unsigned long long m = mm; m; m &= m - 1) W.pl[off++] = (uint16_t)((lane << 6) | (__ffsll((long long)m) - 1));
-    __syncwarp();
-    for (uint32_t p = lane; p < total; p += 32) {
-        const uint32_t e = W.pl[p];
-        const int t = (int)(e & 63);
-        const uint32_t oo = W.lo[0][e >> 6];
-        atomicMin(&W.best[t], parent_key(s_tk[t], oo & kIdMask, ow, oo >> 31));
+    constexpr uint32_t kCap = 2 * kMultiCap;
+    for (uint32_t r0 = 0; r0 < total; r0 += kCap) {
+        uint32_t off = incl - cnt;
+        for (unsigned long long m = mm; m; m &= m - 1) {
+            if (off >= r0 + kCap) break;
+            if (off >= r0) pl[off - r0] = (uint16_t)((lane << 6) | (__ffsll((long long)m) - 1));
+            off++;
+        }
+        __syncwarp();
+        const uint32_t nr = min(total - r0, kCap);
+        for (uint32_t p = lane; p < nr; p += 32) {
+            const uint32_t e = pl[p];
+            const int t = (int)(e & 63);
+            const uint32_t oo = W.lo[0][e >> 6];
+            atomicMin(&W.best[t], parent_key(s_tk[t], oo & kIdMask, ow, oo >> 31));
+        }
+        __syncwarp();
     }
-    __syncwarp();
     p0 = key_to_par(W.best[lane]);
     p1 = key_to_par(W.best[lane + 32]);
     __syncwarp();
@@ -367,7 +406,7 @@ __global__ void k_ms_roots(MsParams P) {
 //   phase C  (only if a hub discovered something) hubs' parents appended,
 //            then one more barrier.
 // ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(kBlock, 3) k_msbfs(MsParams P) {
+__global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
     cg::grid_group grid = cg::this_grid();
     __shared__ uint64_t s_tk[kMsBatch];
     __shared__ uint32_t s_cnt[kMsBatch], s_pos[kMsBatch], s_base[kMsBatch];
