@@ -460,9 +460,44 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
     const int lane = threadIdx.x & 31;
     const int64_t gwarp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
     for (int L = maxd; L >= 1; L--) {
         load_level(P, L, T, s_depth);
         const unsigned long long total = T.soff[B];
+        if constexpr (!kDescent) {
+            // kILP independent vertices per thread: their queue words, their
+            // own sizes and the adds to their parents are in flight together
+            constexpr int kILP = 4;
+            for (unsigned long long base = gtid; base < total; base += kILP * nthr) {
+                size_t qi[kILP], nbk[kILP];
+                uint32_t w[kILP], p[kILP], sz[kILP];
+                bool ok[kILP];
+#pragma unroll
+                for (int k = 0; k < kILP; k++) {
+                    const unsigned long long i = base + (unsigned long long)k * nthr;
+                    ok[k] = i < total;
+                    if (ok[k]) {
+                        const int b = tree_of(T, B, i);
+                        nbk[k] = (size_t)b * P.n;
+                        qi[k] = nbk[k] + T.vb[b] + (uint32_t)(i - T.soff[b]);
+                        w[k] = __ldcg(P.qv + qi[k]);
+                        p[k] = __ldcg(P.parq + qi[k]) & kIdMask;
+                    }
+                }
+#pragma unroll
+                for (int k = 0; k < kILP; k++)
+                    if (ok[k]) sz[k] = 1 + __ldcg(P.size + nbk[k] + w[k]);
+#pragma unroll
+                for (int k = 0; k < kILP; k++) {
+                    if (ok[k]) {
+                        const uint32_t o = atomicAdd(P.size + nbk[k] + p[k], sz[k]);
+                        P.offq[qi[k]] = 1 + o;
+                        P.szq[qi[k]] = sz[k];
+                    }
+                }
+            }
+        } else {
         for (unsigned long long wb = (unsigned long long)gwarp * 32; wb < total;
              wb += (unsigned long long)nwarps * 32) {
             const unsigned long long i = wb + lane;
@@ -492,6 +527,7 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
                 if (valid) P.offq[qi] = 1 + o;
             }
             if (valid) P.szq[qi] = sz;
+        }
         }
         grid.sync();
     }
