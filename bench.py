@@ -46,6 +46,7 @@ def parse():
     ap.add_argument("--walk", type=int, default=0)
     ap.add_argument("--batch", type=int, default=0)
     ap.add_argument("--sub", type=int, default=0, help="trees per labelling launch (0 = auto)")
+    ap.add_argument("--opt", action="append", default=[], help="library option key=value (gb_set_option)")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample-trees", type=int, default=0)
@@ -219,6 +220,9 @@ def main():
     graphb.set_option("walk", args.walk)
     graphb.set_option("batch", args.batch)
     graphb.set_option("sub", args.sub)
+    for kv in args.opt:
+        k, v = kv.split("=")
+        graphb.set_option(k, int(v))
     graphb.load_graph(g)
     n, m, ncomp = graphb.graph_info()
     c_nt = m - n + ncomp

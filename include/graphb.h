@@ -98,7 +98,12 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
  * "cycle_group" trees per cycle-kernel pass (0 = auto), "walk"
  * (0 = two-ended interval walk, 1 = Alg. 3 descent with warp ballots),
  * "timing" (1 = record per-phase CUDA events), "graphs" (1 = CUDA graphs),
- * "sub" (trees per labelling launch, 0 = auto), "msprof" (see gb_msbfs_profile). */
+ * "sub" (trees per labelling launch, 0 = auto), "msprof" (see gb_msbfs_profile),
+ * "recpass" (walk 0: 1 = pre-indexed records scattered in a pass after the
+ * top-down pass, 0 = inside it), "jump" (walk 0: 1, 2 or 4 tree levels per
+ * ancestor record of the cycle walk), "persist" (bytes of an L2 persisting
+ * window over the labelling arrays, 0 = off; sets the device-wide persisting
+ * L2 limit), "reset" (every option back to its default). */
 int gb_set_option(const char *key, int64_t value);
 
 /* Statistics of the last gb_balance / gb_balance_range call:
@@ -130,6 +135,13 @@ int64_t gb_tree_stats(uint64_t *out, int64_t *tree_ids, int64_t max_trees);
  * parent pass, 3 end of the hub pass (0 = not reached).  out has 1024 entries.
  * GB_ESTATE if the option is not set. */
 int gb_msbfs_profile(uint64_t *out);
+
+/* Alg. 4 level profile of the last labelling launch (option "msprof" set):
+ * out[4*L + k], level L < 256: k = 0 globaltimer (ns) at the start of level L
+ * of the bottom-up pass, 1 the same for the top-down pass (level maxd + 1 =
+ * the end), 2 vertices on level L summed over the launch's trees.  out has
+ * 1024 entries.  GB_ESTATE if the option is not set. */
+int gb_label_profile(uint64_t *out);
 
 /* Ingest results (§8 a.1), copied to host arrays (any pointer may be NULL):
  * edge_u[m], edge_v[m] (u < v), edge_neg[m] (1 = negative) indexed by eid;

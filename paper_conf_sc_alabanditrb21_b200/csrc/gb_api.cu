@@ -52,6 +52,9 @@ struct Options {
     int64_t timing = 0;
     int64_t sub = 0;         // trees per labelling launch (0 = auto)
     int64_t msprof = 0;      // record BFS phase timestamps (gb_msbfs_profile)
+    int64_t recpass = 1;     // walk 0: pre-indexed records scattered after the top-down pass
+    int64_t persist = 0;     // bytes of L2 persisting window over the labelling arrays (0 = off)
+    int64_t jump = 1;        // walk 0: levels per ancestor record of the cycle walk (1, 2, 4)
 };
 
 struct Stats {
@@ -85,7 +88,8 @@ static void free_ws(Workspace &w) {
     void *ptrs[] = {w.vst, w.qv, w.qs, w.qr, w.pkeyq, w.lvl, w.vbase, w.size, w.sz64,
                     w.parq, w.offq, w.szq, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
-                    w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof};
+                    w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof,
+                    w.jrec};
     for (void *p : ptrs) if (p) cudaFree(p);
     w = Workspace();
 }
@@ -206,18 +210,20 @@ static int auto_batch(int64_t ntrees) {
     return (int)std::max<int64_t>(b, 1);
 }
 
-// trees per labelling launch: large graphs keep one or two trees' random-access
-// arrays (40-80 MB each) L2-resident; small graphs label the whole batch
+// trees per labelling launch: large graphs label one tree at a time so its
+// random-access array (40 MB for a 10M-vertex tree) stays L2-resident
+// (measured on C3: 1 tree 38.9 ms / 100 trees top-down, 2 trees 49.5, 4 trees
+// 58.4); small graphs label the whole batch
 static int auto_sub(int B) {
     if (S.opt.sub > 0) return (int)std::min<int64_t>(S.opt.sub, B);
-    if (S.g.n >= (1 << 22)) return std::min(B, 2);
+    if (S.g.n >= (1 << 22)) return 1;
     return B;
 }
 
 static int auto_group(int B) {
     if (S.opt.cycle_group > 0) return (int)std::min<int64_t>(S.opt.cycle_group, B);
     // keep the labels of the trees walked together L2-resident (~48 MB)
-    double per = 12.0 * (double)S.g.n;
+    double per = (4.0 + 8.0 * (S.opt.walk == 0 ? S.opt.jump : 1)) * (double)S.g.n;
     int g = (int)std::max(1.0, std::floor(48.0e6 / per));
     return std::max(1, std::min(g, B));
 }
@@ -236,9 +242,22 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     int rc = ensure_workspace(B, descent);
     if (rc) return rc;
     const int G = auto_group(B);
-    if (S.opt.msprof && !S.ws.msprof) GB_CUDA_TRY(cudaMalloc(&S.ws.msprof, sizeof(unsigned long long) * 1024));
+    const int jump = descent ? 1 : (int)S.opt.jump;
+    if (jump > 1 && S.ws.jrec_cap < G * jump) {
+        if (S.ws.jrec) cudaFree(S.ws.jrec);
+        S.ws.jrec = nullptr;
+        S.ws.jrec_cap = 0;
+        cudaError_t e = cudaMalloc(&S.ws.jrec, sizeof(uint2) * (size_t)G * jump * S.g.n);
+        if (e != cudaSuccess) {
+            set_error(std::string("cudaMalloc jrec: ") + cudaGetErrorString(e));
+            S.ws.jrec = nullptr;
+            return e == cudaErrorMemoryAllocation ? GB_ENOMEM : GB_ECUDA;
+        }
+        S.ws.jrec_cap = G * jump;
+    }
+    if (S.opt.msprof && !S.ws.msprof) GB_CUDA_TRY(cudaMalloc(&S.ws.msprof, sizeof(unsigned long long) * 2048));
     if (!S.opt.msprof && S.ws.msprof) { cudaFree(S.ws.msprof); S.ws.msprof = nullptr; }
-    if (S.ws.msprof) GB_CUDA_TRY(cudaMemsetAsync(S.ws.msprof, 0, sizeof(unsigned long long) * 1024, st));
+    if (S.ws.msprof) GB_CUDA_TRY(cudaMemsetAsync(S.ws.msprof, 0, sizeof(unsigned long long) * 2048, st));
     T.batch_used = B;
     T.group_used = G;
     if (!S.d_rec_stats) {
@@ -262,10 +281,11 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 3 * nb, st));
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
-        rc = run_batch_tree(S.g, S.ws, nb, nullptr, st, &T.launches, ev, descent, auto_sub(nb));
+        rc = run_batch_tree(S.g, S.ws, nb, nullptr, st, &T.launches, ev, descent, auto_sub(nb),
+                            (int)S.opt.recpass, (size_t)S.opt.persist);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
-        rc = run_batch_cycles(S.g, S.ws, nb, G, descent, st, &T.launches);
+        rc = run_batch_cycles(S.g, S.ws, nb, G, descent, st, &T.launches, jump);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[5], st));
         rc = run_batch_accumulate(S.g, S.ws, nb, d_cnt, d_agree, st, &T.launches);
@@ -474,6 +494,23 @@ int gb_set_option(const char *key, int64_t value) {
     else if (!strcmp(key, "timing")) S.opt.timing = value != 0;
     else if (!strcmp(key, "sub")) { if (value < 0) return GB_EINVAL; S.opt.sub = value; }
     else if (!strcmp(key, "msprof")) S.opt.msprof = value != 0;
+    else if (!strcmp(key, "reset")) S.opt = Options();
+    else if (!strcmp(key, "recpass")) S.opt.recpass = value != 0;
+    else if (!strcmp(key, "jump")) {
+        if (value != 1 && value != 2 && value != 4) { set_error("jump must be 1, 2 or 4"); return GB_EINVAL; }
+        S.opt.jump = value;
+    }
+    else if (!strcmp(key, "persist")) {
+        if (value < 0) return GB_EINVAL;
+        if (value > 0) {
+            int dev = 0, maxp = 0;
+            GB_CUDA_TRY(cudaGetDevice(&dev));
+            GB_CUDA_TRY(cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev));
+            value = std::min<int64_t>(value, maxp);
+            GB_CUDA_TRY(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)value));
+        }
+        S.opt.persist = value;
+    }
     else if (!strcmp(key, "graphs")) { /* reserved */ }
     else { set_error(std::string("unknown option ") + key); return GB_EINVAL; }
     return GB_OK;
@@ -577,6 +614,12 @@ int gb_get_stats(int64_t *ints, int n_ints, double *phase_ms, int n_phase) {
 int gb_msbfs_profile(uint64_t *out) {
     if (!S.ws.msprof) { set_error("msprof option not set"); return GB_ESTATE; }
     GB_CUDA_TRY(cudaMemcpy(out, S.ws.msprof, sizeof(uint64_t) * 1024, cudaMemcpyDeviceToHost));
+    return GB_OK;
+}
+
+int gb_label_profile(uint64_t *out) {
+    if (!S.ws.msprof) { set_error("msprof option not set"); return GB_ESTATE; }
+    GB_CUDA_TRY(cudaMemcpy(out, S.ws.msprof + 1024, sizeof(uint64_t) * 1024, cudaMemcpyDeviceToHost));
     return GB_OK;
 }
 

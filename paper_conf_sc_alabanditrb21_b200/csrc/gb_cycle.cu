@@ -40,6 +40,7 @@ struct CycleParams {
     unsigned long long *tstat;  // [B][3] {sum cycle length, cycles, state signature}
     int64_t words;
     int b0, G;             // trees b0 .. b0+G-1 of the batch
+    uint2 *jrec;           // [G][n][K] K-level ancestor records (walk 0, option "jump" = K > 1)
 };
 
 constexpr int kCycleBlock = 256;
@@ -136,6 +137,113 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_two_ended(CycleParams P)
             const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
             if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
             // per-tree cycle statistics and state signature
+            warp_stats(lane, g, k, cyc, flip != 0, e, s_k, s_c, s_sig);
+        }
+    }
+    __syncthreads();
+    flush_stats(P, s_k, s_c, s_sig);
+}
+
+// ---------------------------------------------------------------------------
+// K-level records for the two-ended walk (option "jump"): jrec[x][j] =
+// rec[a_j(x)], a_0 = x, a_{j+1} = parent of a_j (the root is its own parent).
+// Built by one streaming pass in pre order -- consecutive pre IDs share most
+// ancestors, so the gathers of rec[a_j] hit L1/L2 -- and written as full
+// 32-byte sectors.  A climb step then still visits every tree edge of the
+// cycle (its sign and range are in the record) but one gather serves K
+// levels: the dependent-load chain of a cycle shrinks by a factor of K.
+// ---------------------------------------------------------------------------
+template <int K>
+__global__ void k_build_jump(const uint2 *__restrict__ rec, uint2 *__restrict__ jrec, int64_t n) {
+    const int g = blockIdx.y;
+    const uint2 *r = rec + (size_t)g * n;
+    uint4 *out = reinterpret_cast<uint4 *>(jrec + (size_t)g * n * K);
+    for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n;
+         x += (int64_t)gridDim.x * blockDim.x) {
+        uint2 a[K];
+        a[0] = __ldg(r + x);
+#pragma unroll
+        for (int j = 1; j < K; j++) a[j] = __ldg(r + (a[j - 1].x & kIdMask));
+#pragma unroll
+        for (int j = 0; j < K; j += 2) out[x * (K / 2) + j / 2] = make_uint4(a[j].x, a[j].y, a[j + 1].x, a[j + 1].y);
+    }
+}
+
+template <int K>
+__device__ __forceinline__ void load_jump(const uint2 *jrec, uint32_t x, uint2 (&a)[K]) {
+    const uint4 *p = reinterpret_cast<const uint4 *>(jrec + (size_t)x * K);
+#pragma unroll
+    for (int j = 0; j < K; j += 2) {
+        const uint4 q = __ldg(p + j / 2);
+        a[j] = make_uint2(q.x, q.y);
+        a[j + 1] = make_uint2(q.z, q.w);
+    }
+}
+
+// one step up from a[0] (the current vertex); the window shifts by one and is
+// refilled from the new vertex's record once it is used up
+template <int K>
+__device__ __forceinline__ void climb_step(const uint2 *jrec, uint2 (&a)[K], int &left, uint32_t &x,
+                                           uint32_t &c) {
+    c ^= a[0].x;
+    x = a[0].x & kIdMask;
+    if (--left == 0) {
+        load_jump<K>(jrec, x, a);
+        left = K;
+    } else {
+#pragma unroll
+        for (int j = 0; j + 1 < K; j++) a[j] = a[j + 1];
+    }
+}
+
+template <int K>
+__global__ void __launch_bounds__(kCycleBlock) k_cycles_jump(CycleParams P) {
+    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup], s_sig[kMaxGroup];
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; s_sig[i] = 0; }
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t word = gw; word < P.words; word += nw) {
+        const int64_t e = word * 32 + lane;
+        const bool valid = e < P.m;
+        uint2 ed = valid ? __ldg(P.edges + e) : make_uint2(0, 0);
+        const uint32_t u = ed.x, v = ed.y & kIdMask, nege = ed.y >> 31;
+        for (int g = 0; g < P.G; g++) {
+            const size_t nb = (size_t)(P.b0 + g) * P.n;
+            const uint2 *jr = P.jrec + (size_t)g * P.n * K;
+            uint32_t flip = 0, k = 0;
+            bool cyc = false;
+            if (valid) {
+                const uint32_t x0 = __ldg(P.pp + nb + u) & kIdMask;
+                const uint32_t y0 = __ldg(P.pp + nb + v) & kIdMask;
+                uint2 ax[K], ay[K];
+                load_jump<K>(jr, x0, ax);
+                load_jump<K>(jr, y0, ay);
+                // tree edge iff one endpoint is the other's parent (simple graph)
+                if ((ax[0].x & kIdMask) != y0 && (ay[0].x & kIdMask) != x0) {
+                    cyc = true;
+                    uint32_t x = x0, y = y0, c = 0;
+                    int lx = K, ly = K;
+                    k = 1;
+                    bool fx = is_anc(x, ax[0].y, y0), fy = is_anc(y, ay[0].y, x0);
+                    while (!(fx && fy)) {
+                        if (!fx) {
+                            climb_step<K>(jr, ax, lx, x, c);
+                            k++;
+                            fx = is_anc(x, ax[0].y, y0);
+                        }
+                        if (!fy) {
+                            climb_step<K>(jr, ay, ly, y, c);
+                            k++;
+                            fy = is_anc(y, ay[0].y, x0);
+                        }
+                    }
+                    flip = (c >> 31) ^ nege;
+                }
+            }
+            const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
+            if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
             warp_stats(lane, g, k, cyc, flip != 0, e, s_k, s_c, s_sig);
         }
     }
@@ -266,8 +374,10 @@ static unsigned grid_cap(int64_t work, int threads, int sms, int per_sm) {
 }
 
 int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool descent,
-                     cudaStream_t st, int64_t *launches) {
+                     cudaStream_t st, int64_t *launches, int jump) {
     CycleParams P;
+    if (descent || !ws.jrec) jump = 1;
+    P.jrec = ws.jrec;
     P.edges = g.edges; P.n = g.n; P.m = g.m;
     P.pp = ws.pp; P.rec = ws.rec; P.crec = ws.crec; P.clist = ws.clist;
     P.fbits = ws.fbits; P.tstat = ws.tstat;
@@ -278,7 +388,15 @@ int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool desce
         P.b0 = b0;
         P.G = std::min(group, B - b0);
         unsigned grid = grid_cap(P.words * 32, kCycleBlock, g.num_sms, 8);
+        if (jump > 1) {
+            const unsigned bx = grid_cap(g.n, 256, g.num_sms, std::max(1, 8 / P.G));
+            if (jump == 2) k_build_jump<2><<<dim3(bx, P.G), 256, 0, st>>>(ws.rec + (size_t)b0 * g.n, ws.jrec, g.n);
+            else k_build_jump<4><<<dim3(bx, P.G), 256, 0, st>>>(ws.rec + (size_t)b0 * g.n, ws.jrec, g.n);
+            ++*launches;
+        }
         if (descent) k_cycles_descent<<<grid, kCycleBlock, 0, st>>>(P);
+        else if (jump == 2) k_cycles_jump<2><<<grid, kCycleBlock, 0, st>>>(P);
+        else if (jump == 4) k_cycles_jump<4><<<grid, kCycleBlock, 0, st>>>(P);
         else k_cycles_two_ended<<<grid, kCycleBlock, 0, st>>>(P);
         ++*launches;
     }

@@ -156,6 +156,8 @@ struct Workspace {
     uint32_t *pp = nullptr;    // v: pre | pi<<31  (pi = root-path parity)
     uint2 *rec = nullptr;      // pre: {up pre | neg<<31, size}
     uint32_t *fbits = nullptr; // [B][ceil(m/32)] flip bitmask
+    uint2 *jrec = nullptr;     // [G][n][K] K-level ancestor records of one cycle group (option "jump")
+    int jrec_cap = 0;          // G * K the buffer holds
     // multi-source BFS state (one bit per tree of the batch, internal ids)
     unsigned long long *vis = nullptr;  // [n] trees that reached the vertex
     unsigned long long *fr = nullptr;   // [2][n] frontier of level L / L+1
@@ -223,7 +225,8 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr,
            int64_t *launches);
 
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
-                   cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub);
+                   cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub,
+                   int recpass = 0, size_t persist = 0);
 
 // multi-source BFS of the B <= kMsBatch sampled trees of a batch (roots, BFS
 // levels, min-hash parents); fills the level lists qv / parq, lvl, vbase, depth
@@ -242,7 +245,7 @@ int debug_tree_views(const Graph &g, Workspace &ws, bool descent, int32_t *d_par
                      int32_t *d_dist, int32_t *d_size, cudaStream_t st);
 
 int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool descent,
-                     cudaStream_t st, int64_t *launches);
+                     cudaStream_t st, int64_t *launches, int jump = 1);
 
 int run_batch_accumulate(const Graph &g, Workspace &ws, int B, int32_t *d_cnt,
                          int32_t *d_agree, cudaStream_t st, int64_t *launches);

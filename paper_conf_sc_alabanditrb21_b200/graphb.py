@@ -58,6 +58,7 @@ def lib():
         "gb_get_stats": (i32, [P, i32, P, i32]),
         "gb_tree_stats": (i64, [P, P, i64]),
         "gb_msbfs_profile": (i32, [P]),
+        "gb_label_profile": (i32, [P]),
         "gb_graph_info": (i32, [P, P, P]),
         "gb_graph_debug": (i32, [P, P, P, P, P]),
         "gb_selftest": (i32, []),
@@ -74,7 +75,8 @@ def lib():
 def exported_symbols():
     return ["gb_load_csr", "gb_balance", "gb_free", "gb_balance_range", "gb_tree_debug",
             "gb_balance_given_tree", "gb_set_option", "gb_get_stats", "gb_tree_stats",
-            "gb_graph_info", "gb_graph_debug", "gb_selftest", "gb_last_error", "gb_msbfs_profile"]
+            "gb_graph_info", "gb_graph_debug", "gb_selftest", "gb_last_error", "gb_msbfs_profile",
+            "gb_label_profile"]
 
 
 def _check(rc):
@@ -270,4 +272,19 @@ def msbfs_profile():
             break
         nxt = t[L + 1, 0] if L + 1 < 256 and t[L + 1, 0] else t[L, 3]
         rows.append((L, (t[L, 1] - t[L, 0]) / 1e6, (t[L, 2] - t[L, 1]) / 1e6, (nxt - t[L, 2]) / 1e6))
+    return rows
+
+
+def label_profile():
+    """Per-level Alg. 4 times (ms) of the last labelling launch: list of
+    (level, vertices, bottom-up ms, top-down ms) -- needs set_option("msprof", 1)."""
+    out = np.zeros(1024, dtype=np.uint64)
+    _check(lib().gb_label_profile(_ptr(out)))
+    t = out.reshape(256, 4).astype(np.int64)
+    D = int(np.max(np.nonzero(t[:, 1])[0])) - 1 if t[:, 1].any() else -1
+    rows = []
+    for L in range(D + 1):
+        bu = (t[L - 1, 0] - t[L, 0]) / 1e6 if L >= 1 and t[L, 0] else 0.0   # bottom-up runs D..1
+        td = (t[L + 1, 1] - t[L, 1]) / 1e6
+        rows.append((L, int(t[L, 2]), bu, td))
     return rows

@@ -19,8 +19,7 @@ pytestmark = pytest.mark.gpu
 @pytest.fixture(autouse=True)
 def _reset_options():
     yield
-    for k in ("batch", "cycle_group", "walk", "timing"):
-        graphb.set_option(k, 0)
+    graphb.set_option("reset", 0)
 
 
 def check_cloud(g, T, seed, **opts):
@@ -103,6 +102,15 @@ def test_power_law_hubs_multi_batch(walk):
     """Hubs (Chung-Lu) + several batches + cycle groups smaller than a batch."""
     g = graphgen.chung_lu(20000, 90000, 2500, 0.75, 0.25, 3)
     check_cloud(g, 37, 11, batch=16, cycle_group=5, walk=walk)
+
+
+@pytest.mark.parametrize("jump,recpass,sub", [(1, 0, 0), (1, 1, 1), (2, 1, 0), (2, 0, 3), (4, 1, 1), (4, 0, 0)])
+def test_walk_records_and_label_passes(jump, recpass, sub):
+    """Walk 0 with 1-, 2- and 4-level ancestor records (option "jump"), the
+    records scattered inside or after the top-down pass ("recpass"), and
+    labelling launches of 1, 3 or all trees ("sub"): all bit-exact."""
+    g = graphgen.chung_lu(30000, 120000, 3000, 0.75, 0.3, 8)
+    check_cloud(g, 21, 3, batch=8, cycle_group=3, jump=jump, recpass=recpass, sub=sub)
 
 
 def test_frustration_cloud_distinct_states():

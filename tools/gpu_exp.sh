@@ -1,1 +1,4 @@
-for sub in 8 64; do timeout 300 python bench.py --config c3 --no-cpu-baseline --no-e2e --sub $sub --steps 3 > gpurun_out/exp_sub$sub.log 2>&1; done
+timeout 600 python -m pytest tests/test_gpu_parity.py -x -q 2>&1 | tail -3
+run() { timeout 300 python bench.py --config $CFG --no-cpu-baseline --no-e2e --steps 3 "$@" 2>&1 | tail -1 | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); print('$CFG $*', round(d['value']/1e9,3), round(d['ms_per_step'],1), {k:round(v,1) for k,v in d['phase_ms_per_step'].items()})" ; }
+for CFG in c3 c2 c4; do run --opt pool=0; run --opt pool=1; done

@@ -1,0 +1,10 @@
+# Round profile: smoke, full C3 bench line, ncu launch list, ncu --set full of the top kernels.
+set -x
+nvidia-smi -L
+python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1; echo smoke $?
+timeout 900 python bench.py > gpurun_out/bench_c3_full.log 2>&1; echo bench $?
+tail -1 gpurun_out/bench_c3_full.log
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_c3.csv python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/ncu_launch.log 2>&1; echo ncu $?
+for k in ${KERNELS:-k_msbfs k_top_down k_cycles_two_ended k_bottom_up}; do
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:$k -c 1 -o gpurun_out/full_$k python tools/prof_run.py c3 64 > gpurun_out/ncu_full_$k.log 2>&1; echo ncufull $k $?
+done
