@@ -124,19 +124,32 @@ class ClockSampler:
 
 
 # ---------------------------------------------------------------------------
-# algorithmic byte model per tree: minimal compulsory
-# traffic of each phase, 4-byte ids / offsets
+# algorithmic byte model per tree (SURVEY.md §8d B_tree): the
+# minimal compulsory traffic of each phase, 4-byte ids / offsets.  Batching
+# (one CSR pass serving B trees) can move less than this; the ncu traffic of
+# the dominant kernel is reported next to it (profiles/traffic_c3.json).
 # ---------------------------------------------------------------------------
 def phase_bytes(n, m, sumk, trees, batch):
-    words = (m + 31) // 32
     return {
-        "init": 4 * n,                                   # dist reset
-        "bfs": 4 * (n + 1) + 24 * m + 12 * n,            # row_ptr, adj+eid+dist per slot, dist+key writes
-        "bottom_up": 32 * n,                             # key, edge, size RMW, parent/off writes
-        "top_down": 32 * n,                              # parent, parent label, offset, size; label writes
-        "cycles": 16 * m + 8 * (sumk / trees) + 4 * words,  # edge table, endpoint labels, k records, flip bits
-        "accumulate": 4 * words + (8 * m + 8 * n) / batch + 4 * n,
+        "init": 0.0,
+        "bfs": 4 * (n + 1) + 8 * m + 8 * m + 8 * n,      # CSR read, one neighbour-state gather per slot, dist+parent
+        "bottom_up": 16 * n,                             # read parent, RMW size
+        "top_down": 16 * n,                              # read parent/size, write pre and the record
+        "cycles": 8 * m + 8 * (sumk / trees),            # non-tree enumeration + one 8 B record per cycle step
+        "accumulate": (m + n) / 8 + 8 * (m + n) / batch,  # flip/pi bits + amortised counter RMW
     }
+
+
+def ncu_traffic(config, kernel, trees_per_launch):
+    """DRAM bytes (read + write) per launch of `kernel` from the committed ncu
+    --set full capture (profiles/traffic_<config>.json), scaled to the trees of
+    one launch here; None if there is no capture for this config/kernel."""
+    try:
+        with open(os.path.join(ROOT, "profiles", f"traffic_{config}.json")) as f:
+            d = json.load(f)[kernel]
+        return d["dram_bytes"] / d["trees"] * trees_per_launch
+    except Exception:
+        return None
 
 
 def load_peaks():
@@ -280,14 +293,24 @@ def main():
     per_tree_sumk = phase["sum_cycle_len"] / max(1, phase["trees"])
     bytes_per_tree = phase_bytes(n, m, per_tree_sumk * phase["trees"], phase["trees"], phase["batch"])
     trees_in_step = phase["trees"]
-    launches_of = {"cycles": max(1, phase["batches"] * -(-phase["batch"] // max(1, phase["cycle_group"])))}
+    sub_trees = 1 if (args.sub == 1 or (args.sub == 0 and n >= (1 << 22))) else phase["batch"]
+    launches_of = {"cycles": max(1, phase["batches"] * -(-phase["batch"] // max(1, phase["cycle_group"]))),
+                   "bottom_up": max(1, -(-trees_in_step // sub_trees)),
+                   "top_down": max(1, -(-trees_in_step // sub_trees))}
     dom_launches = launches_of.get(dom, phase["batches"])
     dom_bytes_per_launch = bytes_per_tree[dom] * trees_in_step / dom_launches
     dom_ms_per_launch = ph[dom] / dom_launches
     peak, peak_src = load_peaks()
     achieved = dom_bytes_per_launch / (dom_ms_per_launch / 1000.0) / 1e9
+    kernel_of = {"bfs": "k_msbfs", "bottom_up": "k_bottom_up", "top_down": "k_top_down",
+                 "cycles": "k_cycles_two_ended", "accumulate": "k_accumulate_edges", "init": "k_ms_roots"}
+    traffic = ncu_traffic(args.config, kernel_of[dom], trees_in_step / dom_launches)
+    path_bytes = sum(bytes_per_tree.values()) * total_trees * args.steps / world
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak, "traffic": None, "peak_source": peak_src,
+                "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                "kernel_name": kernel_of[dom], "trees_per_launch": trees_in_step / dom_launches,
+                "path_achieved": path_bytes / (ms_max / 1000.0) / 1e9,
+                "path_frac": path_bytes / (ms_max / 1000.0) / 1e9 / peak,
                 "bytes_per_launch": dom_bytes_per_launch, "launch_ms": dom_ms_per_launch,
                 "phase_share": {k: v / max(1e-9, sum(ph.values())) for k, v in ph.items()}}
 

@@ -408,6 +408,19 @@ __device__ __forceinline__ unsigned long long gtimer_ns() {
     return t;
 }
 
+// queue-order streams of the level passes: read / written once per pass, so
+// (option GB_LABEL_HINT) they are marked evict_first and leave L2 to the one
+// random-access label array of the pass
+#ifdef GB_LABEL_HINT
+#define GB_QLD(ptr) ld_hint((ptr), qpol)
+#define GB_QST(ptr, val) st_hint((ptr), (val), qpol)
+#define GB_QPOL const uint64_t qpol = l2_stream_policy()
+#else
+#define GB_QLD(ptr) __ldcg(ptr)
+#define GB_QST(ptr, val) (*(ptr) = (val))
+#define GB_QPOL
+#endif
+
 __device__ __forceinline__ int tree_of(const LevelTable &T, int B, unsigned long long i) {
     int lo = 0, hi = B;  // soff[lo] <= i < soff[hi]
     while (hi - lo > 1) {
@@ -482,6 +495,7 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
             // kILP independent vertices per thread: their queue words, their
             // own sizes and the adds to their parents are in flight together
             constexpr int kILP = 4;
+            GB_QPOL;
             for (unsigned long long base = gtid; base < total; base += kILP * nthr) {
                 size_t qi[kILP], nbk[kILP];
                 uint32_t w[kILP], p[kILP], sz[kILP];
@@ -494,8 +508,8 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
                         const int b = tree_of(T, B, i);
                         nbk[k] = (size_t)b * P.n;
                         qi[k] = nbk[k] + T.vb[b] + (uint32_t)(i - T.soff[b]);
-                        w[k] = __ldcg(P.qv + qi[k]);
-                        p[k] = __ldcg(P.parq + qi[k]) & kIdMask;
+                        w[k] = GB_QLD(P.qv + qi[k]);
+                        p[k] = GB_QLD(P.parq + qi[k]) & kIdMask;
                     }
                 }
 #pragma unroll
@@ -505,8 +519,8 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
                 for (int k = 0; k < kILP; k++) {
                     if (ok[k]) {
                         const uint32_t o = atomicAdd(P.size + nbk[k] + p[k], sz[k]);
-                        P.offq[qi[k]] = 1 + o;
-                        P.szq[qi[k]] = sz[k];
+                        GB_QST(P.offq + qi[k], 1 + o);
+                        GB_QST(P.szq + qi[k], sz[k]);
                     }
                 }
             }
@@ -578,6 +592,7 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
             // kILP independent vertices per thread per iteration: their queue
             // words, then their parents' labels, are in flight together
             constexpr int kILP = 4;
+            GB_QPOL;
             for (unsigned long long base = gtid; base < total; base += kILP * nthr) {
                 size_t qi[kILP], nbk[kILP];
                 uint32_t x[kILP], pq[kILP], off[kILP], szx[kILP], ppp[kILP];
@@ -590,10 +605,10 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
                         bk[k] = tree_of(T, B, i);
                         nbk[k] = (size_t)bk[k] * P.n;
                         qi[k] = nbk[k] + T.vb[bk[k]] + (uint32_t)(i - T.soff[bk[k]]);
-                        x[k] = __ldcg(P.qv + qi[k]);
-                        pq[k] = __ldcg(P.parq + qi[k]);
-                        off[k] = __ldcg(P.offq + qi[k]);
-                        szx[k] = __ldcg(P.szq + qi[k]);
+                        x[k] = GB_QLD(P.qv + qi[k]);
+                        pq[k] = GB_QLD(P.parq + qi[k]);
+                        off[k] = GB_QLD(P.offq + qi[k]);
+                        szx[k] = GB_QLD(P.szq + qi[k]);
                     }
                 }
 #pragma unroll
@@ -607,8 +622,8 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
                     const uint32_t pi = (ppp[k] & kNegBit) ^ neg;
                     P.pp[nbk[k] + x[k]] = pre | pi;
                     if (P.recpass) {
-                        P.parq[qi[k]] = up | neg;
-                        P.offq[qi[k]] = pre;
+                        GB_QST(P.parq + qi[k], up | neg);
+                        GB_QST(P.offq + qi[k], pre);
                     } else {
                         P.rec[nbk[k] + pre] = make_uint2(up | neg, szx[k]);
                     }

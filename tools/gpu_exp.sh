@@ -1,4 +1,3 @@
-timeout 600 python -m pytest tests/test_gpu_parity.py -x -q 2>&1 | tail -3
-run() { timeout 300 python bench.py --config $CFG --no-cpu-baseline --no-e2e --steps 3 "$@" 2>&1 | tail -1 | python -c "
-import json,sys; d=json.loads(sys.stdin.read()); print('$CFG $*', round(d['value']/1e9,3), round(d['ms_per_step'],1), {k:round(v,1) for k,v in d['phase_ms_per_step'].items()})" ; }
-for CFG in c3 c2 c4; do run --opt pool=0; run --opt pool=1; done
+for k in k_rec_scatter k_top_down k_bottom_up; do
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:$k -s 3 -c 1 -o gpurun_out/s1_$k python tools/prof_run.py c3 8 > gpurun_out/ncu_s1_$k.log 2>&1; echo $k $?
+done
