@@ -446,8 +446,6 @@ int gb_load_csr(int64_t n, int64_t m, const int64_t *row_ptr, const int32_t *col
     if (rc) { gb_free(); return rc; }
     if (S.ws.B && (S.g.n != old_n || S.g.m != old_m || S.g.ncomp != old_c || S.g.nmulti != old_h))
         free_ws(S.ws);
-    S.h_comp.resize(n);
-    GB_CUDA_TRY(cudaMemcpy(S.h_comp.data(), S.g.comp, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
     {
         size_t freeb = 0, totb = 0;
         GB_CUDA_TRY(cudaMemGetInfo(&freeb, &totb));
@@ -582,6 +580,10 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip, uint64_t *sum_cy
     if (!S.loaded) { set_error("no graph loaded"); return GB_ESTATE; }
     if (!parent) { set_error("NULL parent"); return GB_EINVAL; }
     const int64_t n = S.g.n;
+    if ((int64_t)S.h_comp.size() != n) {   // component of every vertex, copied once per graph
+        S.h_comp.resize(n);
+        GB_CUDA_TRY(cudaMemcpy(S.h_comp.data(), S.g.comp, sizeof(int32_t) * n, cudaMemcpyDeviceToHost));
+    }
     std::vector<int32_t> roots(S.g.ncomp, 0);
     for (int64_t v = 0; v < n; v++) {
         if (parent[v] == -1) roots[S.h_comp[v]]++;

@@ -271,6 +271,57 @@ __global__ void k_cc_rank(const uint32_t *__restrict__ root, const uint32_t *__r
         comp[v] = (int32_t)rank[root[v]];
 }
 
+// Components grouped on the device: a stable radix sort of (comp, v) lists
+// every component's vertices in ascending order; a component starts where the
+// sorted key changes.  The largest component (ties to the smaller rank) is a
+// 64-bit atomicMax of (size << 32 | ~rank).
+__global__ void k_comp_keys(const int32_t *__restrict__ comp, int64_t n, uint32_t *__restrict__ keys,
+                            uint32_t *__restrict__ ids) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        keys[v] = (uint32_t)comp[v];
+        ids[v] = (uint32_t)v;
+    }
+}
+
+__global__ void k_comp_offsets(const uint32_t *__restrict__ skeys, int64_t n, int64_t nc,
+                               int32_t *__restrict__ coff) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t k = skeys[i];
+        if (i == 0 || skeys[i - 1] != k) coff[k] = (int32_t)i;
+        if (i == 0) coff[nc] = (int32_t)n;
+    }
+}
+
+__global__ void k_comp_big(const int32_t *__restrict__ coff, int64_t nc, unsigned long long *big) {
+    unsigned long long best = 0;
+    for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < nc;
+         c += (int64_t)gridDim.x * blockDim.x) {
+        const unsigned long long sz = (unsigned long long)(coff[c + 1] - coff[c]);
+        best = max(best, (sz << 32) | (0xFFFFFFFFull - (unsigned long long)c));
+    }
+    if (best) atomicMax(big, best);
+}
+
+// work items of the multi-source BFS: chunks of <= kChunk slots of every
+// vertex heavier than kLight (internal ids 0 .. nlight0-1, degree-sorted)
+__global__ void k_item_counts(const uint32_t *__restrict__ brow, int64_t nlight0, uint32_t *__restrict__ cnt) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nlight0;
+         i += (int64_t)gridDim.x * blockDim.x)
+        cnt[i] = (brow[i + 1] - brow[i] + (uint32_t)kChunk - 1) / (uint32_t)kChunk;
+}
+
+__global__ void k_item_fill(const uint32_t *__restrict__ brow, const uint32_t *__restrict__ start,
+                            int64_t nlight0, uint2 *__restrict__ items) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < nlight0;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t s0 = brow[i], s1 = brow[i + 1];
+        uint32_t o = start[i];
+        for (uint32_t s = s0; s < s1; s += (uint32_t)kChunk) items[o++] = make_uint2((uint32_t)i, s);
+    }
+}
+
 // ---------------------------------------------------------------------------
 // Degree-sorted view for the multi-source BFS (gb_msbfs.cu)
 // ---------------------------------------------------------------------------
@@ -408,27 +459,41 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
     k_cc_rank<<<grid_for(n, 256, sms), 256, 0, st>>>(ebase, rank, n, g.comp);
     ++*launches;
     {
-        // component offsets and ascending member lists: a counting sort of the
-        // n labels on the host (one-off, O(n))
-        std::vector<int32_t> hc(n);
-        ING_TRY(cudaMemcpyAsync(hc.data(), g.comp, sizeof(int32_t) * n, cudaMemcpyDeviceToHost, st));
+        // component offsets and ascending member lists (device sort, no host pass)
+        uint32_t nr[2] = {0, 0};
+        ING_TRY(cudaMemcpyAsync(&nr[0], rank + (n - 1), sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+        ING_TRY(cudaMemcpyAsync(&nr[1], flag + (n - 1), sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
         ING_TRY(cudaStreamSynchronize(st));
-        int64_t nc = 0;
-        for (int64_t v = 0; v < n; v++) nc = std::max<int64_t>(nc, (int64_t)hc[v] + 1);
-        std::vector<int32_t> coff(nc + 1, 0), fill;
-        for (int64_t v = 0; v < n; v++) coff[hc[v] + 1]++;
-        int32_t big = 0;
-        for (int64_t c = 0; c < nc; c++) if (coff[c + 1] > coff[big + 1]) big = (int32_t)c;
-        for (int64_t c = 0; c < nc; c++) coff[c + 1] += coff[c];
-        fill.assign(coff.begin(), coff.end());
-        std::vector<int32_t> cv(n);
-        for (int64_t v = 0; v < n; v++) cv[fill[hc[v]]++] = (int32_t)v;
-        g.ncomp = nc;
-        g.cbig = big;
+        const int64_t nc = (int64_t)nr[0] + nr[1];
+        uint32_t *keys = nullptr, *skeys = nullptr, *ids = nullptr;
+        unsigned long long *big = nullptr;
+        ING_ALLOC(keys, kArCkeys, 3 * n + 8);
+        skeys = keys + n;
+        ids = keys + 2 * n;
+        big = (unsigned long long *)(((uintptr_t)(keys + 3 * n) + 7) & ~(uintptr_t)7);
         ING_ALLOC(g.coff, kArCoff, nc + 1);
-        ING_TRY(cudaMemcpyAsync(g.coff, coff.data(), sizeof(int32_t) * (nc + 1), cudaMemcpyHostToDevice, st));
-        ING_TRY(cudaMemcpyAsync(g.cverts, cv.data(), sizeof(int32_t) * n, cudaMemcpyHostToDevice, st));
+        k_comp_keys<<<grid_for(n, 256, sms), 256, 0, st>>>(g.comp, n, keys, ids);
+        ++*launches;
+        int bits = 1;
+        while (bits < 32 && (1ll << bits) < nc) bits++;
+        size_t sort_bytes = 0;
+        ING_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sort_bytes, keys, skeys, ids, (uint32_t *)g.cverts,
+                                                (int)n, 0, bits, st));
+        char *sort_tmp = nullptr;
+        ING_ALLOC(sort_tmp, kArSortTmp, sort_bytes);
+        ING_TRY(cub::DeviceRadixSort::SortPairs(sort_tmp, sort_bytes, keys, skeys, ids, (uint32_t *)g.cverts,
+                                                (int)n, 0, bits, st));
+        *launches += 4;
+        k_comp_offsets<<<grid_for(n, 256, sms), 256, 0, st>>>(skeys, n, nc, g.coff);
+        ++*launches;
+        ING_TRY(cudaMemsetAsync(big, 0, sizeof(unsigned long long), st));
+        k_comp_big<<<grid_for(nc, 256, sms), 256, 0, st>>>(g.coff, nc, big);
+        ++*launches;
+        unsigned long long hb = 0;
+        ING_TRY(cudaMemcpyAsync(&hb, big, sizeof(hb), cudaMemcpyDeviceToHost, st));
         ING_TRY(cudaStreamSynchronize(st));
+        g.ncomp = nc;
+        g.cbig = (int32_t)(0xFFFFFFFFull - (hb & 0xFFFFFFFFull));
     }
     {
         // degree-sorted view: stable radix sort of the degrees (descending),
@@ -472,22 +537,28 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
         g.nlight0 = (int64_t)hc[0];
         g.nmulti = (int64_t)hc[1];
         // work items: chunks of <= kChunk slots of every vertex heavier than kLight
-        std::vector<uint32_t> hrow((size_t)g.nlight0 + 1);
-        ING_TRY(cudaMemcpyAsync(hrow.data(), g.brow, sizeof(uint32_t) * (g.nlight0 + 1),
-                                cudaMemcpyDeviceToHost, st));
-        ING_TRY(cudaStreamSynchronize(st));
-        std::vector<uint2> it;
-        it.reserve((size_t)g.nlight0 + 16);
-        for (int64_t i = 0; i < g.nlight0; i++) {
-            if (i == g.nmulti) g.nmulti_items = (int64_t)it.size();
-            for (uint32_t s0 = hrow[i]; s0 < hrow[i + 1]; s0 += (uint32_t)kChunk)
-                it.push_back(make_uint2((uint32_t)i, s0));
+        if (g.nlight0 > 0) {
+            k_item_counts<<<grid_for(g.nlight0, 256, sms), 256, 0, st>>>(g.brow, g.nlight0, upc);
+            ++*launches;
+            rc = exclusive_scan_u32(upc, uptr, g.nlight0, tmp, ntmp, st, launches);
+            if (rc) goto done;
+            uint32_t hv[3] = {0, 0, 0};
+            ING_TRY(cudaMemcpyAsync(&hv[0], uptr + (g.nlight0 - 1), sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+            ING_TRY(cudaMemcpyAsync(&hv[1], upc + (g.nlight0 - 1), sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+            if (g.nmulti < g.nlight0)
+                ING_TRY(cudaMemcpyAsync(&hv[2], uptr + g.nmulti, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+            ING_TRY(cudaStreamSynchronize(st));
+            g.nitems = (int64_t)hv[0] + hv[1];
+            g.nmulti_items = g.nmulti < g.nlight0 ? (int64_t)hv[2] : g.nitems;
+        } else {
+            g.nitems = 0;
+            g.nmulti_items = 0;
         }
-        if (g.nmulti == g.nlight0) g.nmulti_items = (int64_t)it.size();
-        g.nitems = (int64_t)it.size();
         ING_ALLOC(g.items, kArItems, g.nitems);
-        if (g.nitems)
-            ING_TRY(cudaMemcpyAsync(g.items, it.data(), sizeof(uint2) * g.nitems, cudaMemcpyHostToDevice, st));
+        if (g.nitems) {
+            k_item_fill<<<grid_for(g.nlight0, 256, sms), 256, 0, st>>>(g.brow, uptr, g.nlight0, g.items);
+            ++*launches;
+        }
         ING_TRY(cudaStreamSynchronize(st));
     }
     g.n = n;

@@ -211,7 +211,7 @@ void set_error(const std::string &msg);
 enum ArenaSlot {
     kArRowPtr64, kArCol, kArSign, kArErr, kArRowPtr, kArAdj, kArAdjEid, kArEdges, kArComp,
     kArCverts, kArUptr, kArUpc, kArEbase, kArScanTmp, kArLab, kArFlag, kArRank, kArCoff,
-    kArBrow, kArBadj, kArBorig, kArBord, kArBrank, kArItems, kArDeg, kArSortTmp,
+    kArBrow, kArBadj, kArBorig, kArBord, kArBrank, kArItems, kArDeg, kArSortTmp, kArCkeys,
     kArSlots
 };
 void *arena(int slot, size_t bytes);   // nullptr on allocation failure (error set)
