@@ -402,6 +402,28 @@ __device__ __forceinline__ void load_level(const TreeParams &P, int L, LevelTabl
     __syncthreads();
 }
 
+// Levels with at most kSolo vertices (the first and last levels of a BFS
+// tree) are processed by block 0 alone: consecutive small levels are
+// separated by __syncthreads instead of grid barriers, and the other blocks
+// skip them (a grid barrier is kept only where a large level follows or
+// precedes).  kSoloLevels bounds the depth for which the level totals are
+// tabulated in shared memory.
+constexpr unsigned long long kSolo = 1024;
+constexpr int kSoloLevels = 64;
+
+__device__ __forceinline__ bool level_tables(const TreeParams &P, int maxd, const int32_t *s_depth,
+                                             unsigned long long *s_tot) {
+    if (maxd >= kSoloLevels) return false;
+    for (int L = threadIdx.x; L <= maxd; L += blockDim.x) {
+        unsigned long long t = 0;
+        for (int b = 0; b < P.B; b++)
+            if (L <= s_depth[b]) t += __ldcg((const unsigned long long *)(P.lvl + b * P.ls + L)) >> 32;
+        s_tot[L] = t;
+    }
+    __syncthreads();
+    return true;
+}
+
 __device__ __forceinline__ unsigned long long gtimer_ns() {
     unsigned long long t;
     asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
@@ -480,10 +502,8 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
     __syncthreads();
     const int maxd = __ldcg(P.maxd);
     const int lane = threadIdx.x & 31;
-    const int64_t gwarp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+    __shared__ unsigned long long s_tot[kSoloLevels];
+    const bool solo_ok = level_tables(P, maxd, s_depth, s_tot);
     for (int L = maxd; L >= 1; L--) {
         load_level(P, L, T, s_depth);
         const unsigned long long total = T.soff[B];
@@ -491,6 +511,12 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
             P.prof[4 * L] = gtimer_ns();
             P.prof[4 * L + 2] = total;
         }
+        const bool solo = solo_ok && total <= kSolo;
+        const int64_t gwarp = solo ? (int64_t)(threadIdx.x >> 5) : ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+        const int64_t nwarps = solo ? (int64_t)(blockDim.x >> 5) : ((int64_t)gridDim.x * blockDim.x) >> 5;
+        const int64_t gtid = solo ? (int64_t)threadIdx.x : (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+        const int64_t nthr = solo ? (int64_t)blockDim.x : (int64_t)gridDim.x * blockDim.x;
+        if (!solo || blockIdx.x == 0) {
         if constexpr (!kDescent) {
             // kILP independent vertices per thread: their queue words, their
             // own sizes and the adds to their parents are in flight together
@@ -556,7 +582,11 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
             if (valid) P.szq[qi] = sz;
         }
         }
-        grid.sync();
+        }
+        if (L > 1) {
+            if (solo && s_tot[L - 1] <= kSolo) __syncthreads();
+            else grid.sync();
+        }
     }
     if (P.prof && blockIdx.x == 0 && threadIdx.x == 0) P.prof[0] = gtimer_ns();
 }
@@ -582,12 +612,21 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
     __syncthreads();
     const int maxd = __ldcg(P.maxd);
     const bool one_comp = P.ncomp == 1;
-    const int64_t gtid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int64_t nthr = (int64_t)gridDim.x * blockDim.x;
+    __shared__ unsigned long long s_tot[kSoloLevels];
+    const bool solo_ok = level_tables(P, maxd, s_depth, s_tot);
     for (int L = 0; L <= maxd; L++) {
         load_level(P, L, T, s_depth);
         const unsigned long long total = T.soff[B];
         if (P.prof && blockIdx.x == 0 && threadIdx.x == 0 && L < 255) P.prof[4 * L + 1] = gtimer_ns();
+        const bool solo = solo_ok && total <= kSolo;
+        const int64_t gtid = solo ? (int64_t)threadIdx.x : (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+        const int64_t nthr = solo ? (int64_t)blockDim.x : (int64_t)gridDim.x * blockDim.x;
+        // barrier after level L: block-local between two small levels
+        const bool local_sync = solo && L < maxd && s_tot[L + 1] <= kSolo;
+        if (solo && blockIdx.x != 0) {
+            if (L < maxd && !local_sync) grid.sync();
+            continue;
+        }
         if (!kDescent && L > 0) {
             // kILP independent vertices per thread per iteration: their queue
             // words, then their parents' labels, are in flight together
@@ -634,7 +673,10 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
                     }
                 }
             }
-            grid.sync();
+            if (L < maxd) {
+                if (local_sync) __syncthreads();
+                else grid.sync();
+            }
             continue;
         }
         for (unsigned long long i = gtid; i < total; i += nthr) {
@@ -681,7 +723,10 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
                 else atomicAdd(P.s1 + (size_t)b * P.ncomp + C, 1u);
             }
         }
-        grid.sync();
+        if (L < maxd) {
+            if (local_sync) __syncthreads();
+            else grid.sync();
+        }
     }
     if (P.prof && blockIdx.x == 0 && threadIdx.x == 0 && maxd + 1 < 256) P.prof[4 * (maxd + 1) + 1] = gtimer_ns();
     __syncthreads();
