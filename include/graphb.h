@@ -103,12 +103,17 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
  * top-down pass, 0 = inside it), "jump" (walk 0: 1, 2 or 4 tree levels per
  * ancestor record of the cycle walk), "persist" (bytes of an L2 persisting
  * window over the labelling arrays, 0 = off; sets the device-wide persisting
- * L2 limit), "reset" (every option back to its default). */
+ * L2 limit), "harary" (1 = the Harary sides of every tree come from the
+ * paper's L224 procedure on the GPU -- positive-edge CCs of Sigma_T, collapse,
+ * BFS level parity -- instead of the root parity pi; a slow cross-check,
+ * f.2), "reset" (every option back to its default). */
 int gb_set_option(const char *key, int64_t value);
 
 /* Statistics of the last gb_balance / gb_balance_range call:
  * ints[0] trees, [1] sum of cycle lengths, [2] cycles, [3] kernel launches,
- * [4] batches, [5] max tree depth, [6] batch size used, [7] cycle group used.
+ * [4] batches, [5] max tree depth, [6] batch size used, [7] cycle group used,
+ * [8] edges of some Sigma_T that contradict the L224 bipartition (option
+ * "harary" only; 0 means every balanced state was checked and consistent).
  * phase_ms[GB_NPHASE] (valid when "timing" was 1): summed CUDA-event times.
  * Returns the number of ints written. */
 #define GB_NPHASE 6

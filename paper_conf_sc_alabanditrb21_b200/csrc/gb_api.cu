@@ -54,11 +54,12 @@ struct Options {
     int64_t msprof = 0;      // record BFS phase timestamps (gb_msbfs_profile)
     int64_t recpass = 1;     // walk 0: pre-indexed records scattered after the top-down pass
     int64_t persist = 0;     // bytes of L2 persisting window over the labelling arrays (0 = off)
+    int64_t harary = 0;      // 1: Harary sides by the L224 procedure (gb_harary.cu)
     int64_t jump = 1;        // walk 0: levels per ancestor record of the cycle walk (1, 2, 4)
 };
 
 struct Stats {
-    int64_t trees = 0, launches = 0, batches = 0, batch_used = 0, group_used = 0;
+    int64_t trees = 0, launches = 0, batches = 0, batch_used = 0, group_used = 0, harary_bad = 0;
     uint64_t sumk = 0, cycles = 0;
     int64_t max_depth = 0;
     double phase_ms[GB_NPHASE] = {0};
@@ -76,6 +77,7 @@ struct State {
     int32_t *d_given = nullptr;                    // caller tree (gb_balance_given_tree)
     unsigned long long *d_visited = nullptr;       // [kMaxBatch]
     unsigned long long *d_rec_stats = nullptr;     // [kRecCap][4]
+    unsigned long long *d_hbad = nullptr;          // option "harary": violations found
     std::vector<int32_t> h_comp;
     size_t free_at_load = 0;   // device memory free after ingest (cudaMemGetInfo costs ~2 ms)
     Options opt;
@@ -89,7 +91,7 @@ static void free_ws(Workspace &w) {
                     w.parq, w.offq, w.szq, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
                     w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof,
-                    w.jrec};
+                    w.jrec, w.hlab};
     for (void *p : ptrs) if (p) cudaFree(p);
     w = Workspace();
 }
@@ -288,6 +290,14 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         rc = run_batch_cycles(S.g, S.ws, nb, G, descent, st, &T.launches, jump);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[5], st));
+        if (S.opt.harary) {
+            if (!S.d_hbad) {
+                GB_CUDA_TRY(cudaMalloc(&S.d_hbad, sizeof(unsigned long long)));
+            }
+            if (T.batches == 0) GB_CUDA_TRY(cudaMemsetAsync(S.d_hbad, 0, sizeof(unsigned long long), st));
+            rc = run_batch_harary(S.g, S.ws, nb, st, &T.launches, S.d_hbad);
+            if (rc) return rc;
+        }
         rc = run_batch_accumulate(S.g, S.ws, nb, d_cnt, d_agree, st, &T.launches);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[6], st));
@@ -300,6 +310,12 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         T.batches++;
     }
     GB_CUDA_TRY(cudaGetLastError());
+    if (S.opt.harary) {
+        unsigned long long hb = 0;
+        GB_CUDA_TRY(cudaMemcpyAsync(&hb, S.d_hbad, sizeof(hb), cudaMemcpyDeviceToHost, st));
+        GB_CUDA_TRY(cudaStreamSynchronize(st));
+        T.harary_bad = (int64_t)hb;
+    }
     const int64_t nrec = std::min<int64_t>(K, kRecCap);
     T.per_tree.resize(4 * nrec);
     GB_CUDA_TRY(cudaMemcpyAsync(T.per_tree.data(), S.d_rec_stats, sizeof(uint64_t) * 4 * nrec,
@@ -411,6 +427,7 @@ void gb_free(void) {
     arena_free_all();
     if (S.d_visited) cudaFree(S.d_visited);
     if (S.d_rec_stats) cudaFree(S.d_rec_stats);
+    if (S.d_hbad) cudaFree(S.d_hbad);
     if (S.stream) cudaStreamDestroy(S.stream);
     Options keep = S.opt;
     S = State();
@@ -493,6 +510,7 @@ int gb_set_option(const char *key, int64_t value) {
     else if (!strcmp(key, "sub")) { if (value < 0) return GB_EINVAL; S.opt.sub = value; }
     else if (!strcmp(key, "msprof")) S.opt.msprof = value != 0;
     else if (!strcmp(key, "reset")) S.opt = Options();
+    else if (!strcmp(key, "harary")) S.opt.harary = value != 0;
     else if (!strcmp(key, "recpass")) S.opt.recpass = value != 0;
     else if (!strcmp(key, "jump")) {
         if (value != 1 && value != 2 && value != 4) { set_error("jump must be 1, 2 or 4"); return GB_EINVAL; }
@@ -604,10 +622,10 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip, uint64_t *sum_cy
 
 int gb_get_stats(int64_t *ints, int n_ints, double *phase_ms, int n_phase) {
     const Stats &T = S.st;
-    int64_t v[8] = {T.trees, (int64_t)T.sumk, (int64_t)T.cycles, T.launches, T.batches,
-                    T.max_depth, T.batch_used, T.group_used};
+    int64_t v[9] = {T.trees, (int64_t)T.sumk, (int64_t)T.cycles, T.launches, T.batches,
+                    T.max_depth, T.batch_used, T.group_used, T.harary_bad};
     int k = 0;
-    for (; ints && k < n_ints && k < 8; k++) ints[k] = v[k];
+    for (; ints && k < n_ints && k < 9; k++) ints[k] = v[k];
     for (int i = 0; phase_ms && i < n_phase && i < GB_NPHASE; i++) phase_ms[i] = T.phase_ms[i];
     return k;
 }

@@ -156,6 +156,7 @@ struct Workspace {
     uint32_t *pp = nullptr;    // v: pre | pi<<31  (pi = root-path parity)
     uint2 *rec = nullptr;      // pre: {up pre | neg<<31, size}
     uint32_t *fbits = nullptr; // [B][ceil(m/32)] flip bitmask
+    int32_t *hlab = nullptr;   // option "harary": [3n + 16] CC labels, CC roots, BFS levels, flag
     uint2 *jrec = nullptr;     // [G][n][K] K-level ancestor records of one cycle group (option "jump")
     int jrec_cap = 0;          // G * K the buffer holds
     // multi-source BFS state (one bit per tree of the batch, internal ids)
@@ -249,6 +250,12 @@ int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool desce
 
 int run_batch_accumulate(const Graph &g, Workspace &ws, int B, int32_t *d_cnt,
                          int32_t *d_agree, cudaStream_t st, int64_t *launches);
+
+// f.2: Harary sides of the B trees of a batch by the L224 procedure (replaces
+// the pi bits of pp and the per-component counts s1); d_bad counts edges
+// whose sign contradicts the resulting bipartition
+int run_batch_harary(const Graph &g, Workspace &ws, int B, cudaStream_t st, int64_t *launches,
+                     unsigned long long *d_bad);
 
 int exclusive_scan_u32(const uint32_t *in, uint32_t *out, int64_t count, uint32_t *tmp,
                        size_t tmp_elems, cudaStream_t st, int64_t *launches);

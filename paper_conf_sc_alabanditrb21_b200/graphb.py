@@ -232,11 +232,11 @@ def balance_given_tree(parent):
 
 
 def stats():
-    ints = np.zeros(8, np.int64)
+    ints = np.zeros(9, np.int64)
     ph = np.zeros(len(PHASES), np.float64)
-    lib().gb_get_stats(_ptr(ints), 8, _ptr(ph), len(PHASES))
+    lib().gb_get_stats(_ptr(ints), 9, _ptr(ph), len(PHASES))
     keys = ("trees", "sum_cycle_len", "cycles", "launches", "batches", "max_depth", "batch",
-            "cycle_group")
+            "cycle_group", "harary_violations")
     d = {k: int(v) for k, v in zip(keys, ints)}
     d["phase_ms"] = {k: float(v) for k, v in zip(PHASES, ph)}
     return d

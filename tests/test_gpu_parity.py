@@ -113,6 +113,22 @@ def test_walk_records_and_label_passes(jump, recpass, sub):
     check_cloud(g, 21, 3, batch=8, cycle_group=3, jump=jump, recpass=recpass, sub=sub)
 
 
+@pytest.mark.parametrize("which", ["er", "chung_lu", "forest", "diamond", "planted", "grid"])
+def test_harary_l224_procedure_on_gpu(which):
+    """f.2 (L224): Harary sides from the paper's procedure on the GPU --
+    CCs of the positive edges of Sigma_T, collapse, BFS level parity -- give
+    the same agree counts as the oracle (which runs L224 literally), and every
+    edge of every Sigma_T is consistent with the bipartition (L216)."""
+    g = {"er": lambda: graphgen.er(4000, 16000, 0.3, 6),
+         "chung_lu": lambda: graphgen.chung_lu(20000, 90000, 2500, 0.75, 0.5, 4),
+         "forest": lambda: graphgen.er(5000, 3000, 0.4, 2),
+         "diamond": lambda: graphgen.diamond(),
+         "planted": lambda: graphgen.planted_signs(graphgen.er(3000, 12000, 0.0, 3), 5)[0],
+         "grid": lambda: graphgen.grid2d(40, 50, 0.5, 7)}[which]()
+    st = check_cloud(g, 13, 2, harary=1, batch=5)
+    assert st["harary_violations"] == 0
+
+
 def test_frustration_cloud_distinct_states():
     """f.2 (Fig. 2, L81/L86): distinct nearest balanced states over many
     trees, counted from the per-tree state signatures, equal the oracle's."""
