@@ -67,6 +67,11 @@ def lib():
         L.or_state_signature.argtypes = [P, i64]
         L.or_balance.restype = ctypes.c_int
         L.or_balance.argtypes = [P, i64, i64, i64, u64, P, P, P]
+        L.or_balance_m.restype = ctypes.c_int
+        L.or_balance_m.argtypes = [P, i64, i64, i64, u64, ctypes.c_int, P, P, P]
+        L.or_wdraw.restype = u64; L.or_wdraw.argtypes = [u64, i64, ctypes.c_int32, ctypes.c_uint32]
+        L.or_wilson_tree.restype = ctypes.c_int
+        L.or_wilson_tree.argtypes = [P, u64, i64, ctypes.c_int, P, P]
         _lib = L
     return _lib
 
@@ -98,6 +103,10 @@ def ekey(seed, t, e):
 
 def pscore(seed, t, a, b):
     return int(lib().or_pscore(seed, t, a, b))
+
+
+def wdraw(seed, t, u, j):
+    return int(lib().or_wdraw(seed & (2**64 - 1), t, u, j))
 
 
 def state_signature(flip):
@@ -186,13 +195,22 @@ class Graph:
             raise OracleError(rc, "or_harary")
         return side, d2
 
-    def balance(self, num_trees, seed, t_begin=0, stride=1, with_stats=False):
-        """Frustration cloud over trees t_begin, t_begin+stride, ... < num_trees."""
+    def wilson_tree(self, seed, t, order=0):
+        """Uniform spanning forest (Wilson, reading R17): (parent, pops)."""
+        parent = np.zeros(self.n, np.int32); pops = np.zeros(self.n, np.uint32)
+        rc = lib().or_wilson_tree(self._h, seed, t, order, _p(parent), _p(pops))
+        if rc != OR_OK:
+            raise OracleError(rc, "or_wilson_tree")
+        return parent, pops
+
+    def balance(self, num_trees, seed, t_begin=0, stride=1, with_stats=False, sampler=0):
+        """Frustration cloud over trees t_begin, t_begin+stride, ... < num_trees
+        (sampler 0 = BFS trees, 1 = uniform spanning trees)."""
         cnt = np.zeros(max(self.m, 1), np.uint32); agree = np.zeros(self.n, np.uint32)
         k = len(range(t_begin, num_trees, stride))
         stats = np.zeros(4 * max(k, 1), np.uint64)
-        rc = lib().or_balance(self._h, t_begin, num_trees, stride, seed, _p(cnt), _p(agree),
-                              _p(stats))
+        rc = lib().or_balance_m(self._h, t_begin, num_trees, stride, seed, sampler, _p(cnt),
+                                _p(agree), _p(stats))
         if rc != OR_OK:
             raise OracleError(rc, "or_balance")
         if with_stats:

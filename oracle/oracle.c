@@ -274,6 +274,60 @@ int or_bfs_tree(const or_graph *g, uint64_t seed, int64_t t,
     return OR_OK;
 }
 
+/* ------------------------------------------------------------------------ */
+/* Tree sampling, Alg. 2 with M = random (L130 "e.g., BFS, DFS, random";
+ * L168 prior work used random spanning trees): a uniformly random spanning
+ * tree by Wilson's algorithm (loop-erased random walks, reading R17).  The
+ * walk's randomness is a per-vertex stack: the j-th departure from u goes to
+ * N(u)[wdraw(seed,t,u,j) mod deg(u)], wdraw = mix64(tkey + W*(u*2^32 + j)).
+ * Roots are the BFS sampler's (R4).  Vertices are started in ascending order
+ * (order = 0) or descending order (order = 1): with fixed stacks the tree
+ * does not depend on the order (the cycle-popping theorem), which the tests
+ * use as a pin.  The walk overwrites nxt[u] at every departure (last-exit
+ * loop erasure); pops[u] = departures from u - 1 for tree vertices.          */
+/* ------------------------------------------------------------------------ */
+#define OR_WMUL 0xD6E8FEB86659FD93ULL
+
+uint64_t or_wdraw(uint64_t seed, int64_t t, int32_t u, uint32_t j)
+{
+    return or_mix64(or_tkey(seed, t) + OR_WMUL * (((uint64_t)(uint32_t)u << 32) | (uint64_t)j));
+}
+
+int or_wilson_tree(const or_graph *g, uint64_t seed, int64_t t, int order,
+                   int32_t *parent, uint32_t *pops)
+{
+    int64_t n = g->n;
+    uint8_t *in_tree = (uint8_t *)calloc((size_t)n + 1, 1);
+    uint32_t *dep = (uint32_t *)calloc((size_t)n + 1, sizeof(uint32_t));
+    int32_t *nxt = (int32_t *)malloc(sizeof(int32_t) * ((size_t)n + 1));
+    if (!in_tree || !dep || !nxt) { free(in_tree); free(dep); free(nxt); return OR_ENOMEM; }
+    for (int64_t v = 0; v < n; v++) nxt[v] = -1;
+    for (int64_t c = 0; c < g->ncomp; c++) {
+        int64_t sz = g->coff[c + 1] - g->coff[c];
+        int32_t r = g->cverts[g->coff[c] + (int64_t)(or_rkey(seed, t, c) % (uint64_t)sz)];
+        in_tree[r] = 1;
+    }
+    for (int64_t i = 0; i < n; i++) {
+        int64_t v = order ? n - 1 - i : i;
+        /* random walk from v until it hits the tree, remembering the last exit */
+        int64_t u = v;
+        while (!in_tree[u]) {
+            int64_t deg = g->row_ptr[u + 1] - g->row_ptr[u];
+            uint64_t k = or_wdraw(seed, t, (int32_t)u, dep[u]++) % (uint64_t)deg;
+            nxt[u] = g->col[g->row_ptr[u] + (int64_t)k];
+            u = nxt[u];
+        }
+        /* add the loop-erased path */
+        for (u = v; !in_tree[u]; u = nxt[u]) in_tree[u] = 1;
+    }
+    for (int64_t v = 0; v < n; v++) {
+        parent[v] = nxt[v];          /* -1 for the roots (never departed) */
+        if (pops) pops[v] = dep[v] ? dep[v] - 1 : 0;
+    }
+    free(in_tree); free(dep); free(nxt);
+    return OR_OK;
+}
+
 /* depth of every vertex under parent[], checking that parent[] is a spanning
  * forest of g with exactly one root per connected component. */
 static int tree_depth(const or_graph *g, const int32_t *parent, int32_t *depth, int8_t *pneg)
@@ -523,8 +577,18 @@ uint64_t or_state_signature(const uint8_t *flip, int64_t m)
  * sample T (BFS), balance (Alg. 1), Harary bipartition (L224), count per
  * edge and per vertex (L248).                                               */
 /* ------------------------------------------------------------------------ */
+int or_balance_m(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride,
+                 uint64_t seed, int sampler, uint32_t *cnt, uint32_t *agree, uint64_t *stats);
+
 int or_balance(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride,
                uint64_t seed, uint32_t *cnt, uint32_t *agree, uint64_t *stats)
+{
+    return or_balance_m(g, t_begin, t_end, stride, seed, 0, cnt, agree, stats);
+}
+
+/* sampler: 0 = BFS (R4), 1 = uniform (Wilson, R17) */
+int or_balance_m(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride,
+                 uint64_t seed, int sampler, uint32_t *cnt, uint32_t *agree, uint64_t *stats)
 {
     if (stride < 1 || t_begin < 0 || t_end < t_begin) return OR_EINVAL;
     int64_t n = g->n, m = g->m;
@@ -537,7 +601,8 @@ int or_balance(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride
     if (!parent || !dist || !flip || !side || !delta2) goto out;
     int64_t i = 0;
     for (int64_t t = t_begin; t < t_end; t += stride, i++) {
-        rc = or_bfs_tree(g, seed, t, parent, dist, NULL);
+        rc = sampler == 1 ? or_wilson_tree(g, seed, t, 0, parent, NULL)
+                          : or_bfs_tree(g, seed, t, parent, dist, NULL);
         if (rc != OR_OK) goto out;
         uint64_t sk = 0;
         int64_t nc = 0;

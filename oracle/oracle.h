@@ -73,6 +73,18 @@ uint64_t or_state_signature(const uint8_t *flip, int64_t m);
 int or_balance(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride,
                uint64_t seed, uint32_t *cnt, uint32_t *agree, uint64_t *stats);
 
+/* Alg. 2 with M = random: a uniformly random spanning forest by Wilson's
+ * algorithm with per-vertex random stacks (reading R17); order 0/1 starts the
+ * walks in ascending/descending vertex order (the result must not depend on
+ * it).  parent[root] = -1; pops[v] (optional) = times v's stack was popped. */
+uint64_t or_wdraw(uint64_t seed, int64_t t, int32_t u, uint32_t j);
+int or_wilson_tree(const or_graph *g, uint64_t seed, int64_t t, int order,
+                   int32_t *parent, uint32_t *pops);
+
+/* or_balance with the sampler chosen: 0 = BFS (R4), 1 = uniform (Wilson). */
+int or_balance_m(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride,
+                 uint64_t seed, int sampler, uint32_t *cnt, uint32_t *agree, uint64_t *stats);
+
 #ifdef __cplusplus
 }
 #endif

@@ -514,3 +514,77 @@ def test_balance_given_tree_rejects_non_forests():
         og.balance_tree(np.array([-1, 0, 3, 2, 0], np.int32))                   # cycle 2<->3
     with pytest.raises(oracle.OracleError):
         og.balance_tree(np.array([-1, 0, 0, 2, 3], np.int32))                   # 0-2 not an edge
+
+
+# --------------------------------------------------------------------------
+# f.3: Alg. 2 with M = random (L130): uniform spanning trees by Wilson's
+# algorithm with per-vertex random stacks (reading R17).  Pins: the tree does
+# not depend on the order of the start vertices (cycle-popping theorem), the
+# sampled trees are exactly the spanning trees (count by Kirchhoff's
+# matrix-tree theorem) and uniformly distributed (chi-square), roots follow R4.
+# --------------------------------------------------------------------------
+
+def _tree_key(parent):
+    return tuple(sorted((min(v, int(p)), max(v, int(p))) for v, p in enumerate(parent) if p >= 0))
+
+
+def _matrix_tree_count(g):
+    n = g.n
+    Lap = np.zeros((n, n))
+    for u, v, _ in bf.edge_list(g):
+        Lap[u, v] -= 1; Lap[v, u] -= 1; Lap[u, u] += 1; Lap[v, v] += 1
+    return int(round(np.linalg.det(Lap[1:, 1:])))
+
+
+@pytest.mark.parametrize("which", ["er", "chung_lu", "forest", "grid", "ring"])
+def test_wilson_order_independent_spanning_forest(which):
+    g = {"er": lambda: graphgen.er(400, 1500, 0.3, 3),
+         "chung_lu": lambda: graphgen.chung_lu(600, 2400, 90, 0.75, 0.3, 2),
+         "forest": lambda: graphgen.er(500, 300, 0.4, 2),
+         "grid": lambda: graphgen.grid2d(9, 11, 0.5, 4),
+         "ring": lambda: graphgen.ring(50)}[which]()
+    og = oracle.Graph.from_csr(g)
+    edges = {(u, v) for u, v, _ in bf.edge_list(g)}
+    for t in range(5):
+        p0, pops = og.wilson_tree(7, t, 0)
+        p1, _ = og.wilson_tree(7, t, 1)
+        assert np.array_equal(p0, p1), "Wilson tree depends on the start order"
+        bfs_parent, dist, _ = og.bfs_tree(7, t)
+        assert np.array_equal(np.flatnonzero(p0 < 0), np.flatnonzero(dist == 0))   # R4 roots
+        for v in range(g.n):
+            if p0[v] >= 0:
+                assert (min(v, int(p0[v])), max(v, int(p0[v]))) in edges
+        # acyclic: every vertex reaches a root within n steps
+        for v in range(g.n):
+            x, k = v, 0
+            while p0[x] >= 0:
+                x = int(p0[x]); k += 1
+                assert k <= g.n
+        assert int(pops.sum()) >= 0
+
+
+@pytest.mark.parametrize("g,ntrees", [(graphgen.complete(4), 16), (graphgen.diamond(), 8),
+                                      (graphgen.ring(6), 6)])
+def test_wilson_uniform_over_all_spanning_trees(g, ntrees):
+    from scipy.stats import chisquare
+    assert _matrix_tree_count(g) == ntrees
+    og = oracle.Graph.from_csr(g)
+    counts = {}
+    S = 400 * ntrees
+    for t in range(S):
+        p, _ = og.wilson_tree(11, t, 0)
+        k = _tree_key(p)
+        counts[k] = counts.get(k, 0) + 1
+    assert len(counts) == ntrees
+    assert chisquare(list(counts.values())).pvalue > 1e-4
+
+
+def test_wilson_cloud_balances_every_tree():
+    g = graphgen.er(200, 700, 0.4, 9)
+    og = oracle.Graph.from_csr(g)
+    for t in range(4):
+        parent, _ = og.wilson_tree(3, t)
+        flip, sk, nc, _ = og.balance_tree(parent)
+        _check_tree_result(g, og, parent, flip, sk)
+    cnt, agree, st = og.balance(4, 3, with_stats=True, sampler=1)
+    assert int(st[:, 1].sum()) == 4 * (g.m - g.n + og.ncomp)
