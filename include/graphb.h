@@ -106,7 +106,11 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
  * L2 limit), "harary" (1 = the Harary sides of every tree come from the
  * paper's L224 procedure on the GPU -- positive-edge CCs of Sigma_T, collapse,
  * BFS level parity -- instead of the root parity pi; a slow cross-check,
- * f.2), "reset" (every option back to its default). */
+ * f.2), "sampler" (Alg. 2 method M, L130: 0 = BFS trees (default, reading
+ * R4), 1 = uniform random spanning trees by Wilson's algorithm with
+ * per-vertex random stacks (reading R17), sampled on the GPU by parallel
+ * cycle popping and processed one tree at a time; gb_tree_debug then reports
+ * that tree), "reset" (every option back to its default). */
 int gb_set_option(const char *key, int64_t value);
 
 /* Statistics of the last gb_balance / gb_balance_range call:

@@ -54,6 +54,7 @@ struct Options {
     int64_t msprof = 0;      // record BFS phase timestamps (gb_msbfs_profile)
     int64_t recpass = 1;     // walk 0: pre-indexed records scattered after the top-down pass
     int64_t persist = 0;     // bytes of L2 persisting window over the labelling arrays (0 = off)
+    int64_t sampler = 0;     // Alg. 2 M: 0 BFS (R4), 1 uniform spanning trees (Wilson, R17)
     int64_t harary = 0;      // 1: Harary sides by the L224 procedure (gb_harary.cu)
     int64_t jump = 1;        // walk 0: levels per ancestor record of the cycle walk (1, 2, 4)
 };
@@ -91,7 +92,7 @@ static void free_ws(Workspace &w) {
                     w.parq, w.offq, w.szq, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
                     w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof,
-                    w.jrec, w.hlab};
+                    w.jrec, w.hlab, w.wbuf, w.wparent};
     for (void *p : ptrs) if (p) cudaFree(p);
     w = Workspace();
 }
@@ -205,6 +206,7 @@ __global__ void k_record_stats(const unsigned long long *tstat, const int32_t *d
 }
 
 static int auto_batch(int64_t ntrees) {
+    if (S.opt.sampler == 1) return 1;   // sampled trees go one at a time (caller-tree path)
     if (S.opt.batch > 0) return (int)std::min<int64_t>(S.opt.batch, kMaxBatch);
     const size_t have = S.free_at_load;
     int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk == 1));
@@ -284,7 +286,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
         rc = run_batch_tree(S.g, S.ws, nb, nullptr, st, &T.launches, ev, descent, auto_sub(nb),
-                            (int)S.opt.recpass, (size_t)S.opt.persist);
+                            (int)S.opt.recpass, (size_t)S.opt.persist, (int)S.opt.sampler);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
         rc = run_batch_cycles(S.g, S.ws, nb, G, descent, st, &T.launches, jump);
@@ -351,7 +353,8 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 3, st));
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
-    rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk == 1, 1);
+    rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk == 1, 1,
+                        0, 0, d_given ? 0 : (int)S.opt.sampler);
     if (rc) return rc;
     if (d_given) {
         unsigned long long vis = 0;
@@ -511,6 +514,10 @@ int gb_set_option(const char *key, int64_t value) {
     else if (!strcmp(key, "msprof")) S.opt.msprof = value != 0;
     else if (!strcmp(key, "reset")) S.opt = Options();
     else if (!strcmp(key, "harary")) S.opt.harary = value != 0;
+    else if (!strcmp(key, "sampler")) {
+        if (value != 0 && value != 1) { set_error("sampler must be 0 (BFS) or 1 (uniform)"); return GB_EINVAL; }
+        S.opt.sampler = value;
+    }
     else if (!strcmp(key, "recpass")) S.opt.recpass = value != 0;
     else if (!strcmp(key, "jump")) {
         if (value != 1 && value != 2 && value != 4) { set_error("jump must be 1, 2 or 4"); return GB_EINVAL; }

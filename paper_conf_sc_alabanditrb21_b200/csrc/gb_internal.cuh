@@ -156,6 +156,8 @@ struct Workspace {
     uint32_t *pp = nullptr;    // v: pre | pi<<31  (pi = root-path parity)
     uint2 *rec = nullptr;      // pre: {up pre | neg<<31, size}
     uint32_t *fbits = nullptr; // [B][ceil(m/32)] flip bitmask
+    void *wbuf = nullptr;      // option "sampler" = 1: Wilson state (20n bytes)
+    int32_t *wparent = nullptr;// its tree (parent, -1 at the roots)
     int32_t *hlab = nullptr;   // option "harary": [3n + 16] CC labels, CC roots, BFS levels, flag
     uint2 *jrec = nullptr;     // [G][n][K] K-level ancestor records of one cycle group (option "jump")
     int jrec_cap = 0;          // G * K the buffer holds
@@ -227,7 +229,12 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr,
 
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
                    cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub,
-                   int recpass = 0, size_t persist = 0);
+                   int recpass = 0, size_t persist = 0, int sampler = 0);
+
+// f.3: uniform random spanning forest of tree ws.tkey[0] (Wilson by parallel
+// cycle popping, gb_wilson.cu) -> parent (-1 at the roots)
+int run_wilson(const Graph &g, Workspace &ws, cudaStream_t st, int64_t *launches, int32_t *parent,
+               int64_t *rounds_out);
 
 // multi-source BFS of the B <= kMsBatch sampled trees of a batch (roots, BFS
 // levels, min-hash parents); fills the level lists qv / parq, lvl, vbase, depth

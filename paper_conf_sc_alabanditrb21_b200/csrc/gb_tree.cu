@@ -871,7 +871,7 @@ static int set_window(cudaStream_t st, void *base, size_t bytes, size_t persist)
 
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
                    cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub,
-                   int recpass, size_t persist) {
+                   int recpass, size_t persist, int sampler) {
     if (descent) recpass = 0;
     static int bfs_blocks = 0, up_blocks[2] = {0, 0}, down_blocks[2] = {0, 0};
     if (!bfs_blocks) {
@@ -889,13 +889,24 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
     else GB_CUDA_TRY(cudaMemsetAsync(ws.size, 0, sizeof(uint32_t) * (size_t)B * g.n, st));
     k_batch_prep<<<1, kMaxBatch, 0, st>>>(P);
     ++*launches;
+    // f.3: a uniform random spanning tree (B = 1), then the caller-tree path
+    const bool sampled = sampler == 1 && !given_parent;
+    if (sampled) {
+        if (ev) GB_CUDA_TRY(cudaEventRecord(ev[1], st));
+        if (!ws.wparent) GB_CUDA_TRY(cudaMalloc(&ws.wparent, sizeof(int32_t) * (size_t)g.n));
+        int rc = run_wilson(g, ws, st, launches, ws.wparent, nullptr);
+        if (rc) return rc;
+        given_parent = ws.wparent;
+        P.given = given_parent;
+        P.visited = ws.visited;
+    }
     if (given_parent) {
         // a caller tree (B = 1): push BFS along its parent edges
         GB_CUDA_TRY(cudaMemsetAsync(ws.vst, 0, sizeof(uint32_t) * (size_t)P.nw, st));
         k_roots_given<<<(unsigned)std::min<int64_t>((g.n + 255) / 256, 4096), 256, 0, st>>>(P);
         ++*launches;
         GB_CUDA_TRY(cudaGetLastError());
-        if (ev) GB_CUDA_TRY(cudaEventRecord(ev[1], st));
+        if (ev && !sampled) GB_CUDA_TRY(cudaEventRecord(ev[1], st));
         int rc = launch_coop((const void *)k_bfs, bfs_blocks, P, st);
         if (rc) return rc;
         ++*launches;

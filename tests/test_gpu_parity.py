@@ -30,7 +30,7 @@ def check_cloud(g, T, seed, **opts):
     st = graphb.stats()
     ids, per = graphb.tree_stats()
     og = oracle.Graph.from_csr(g)
-    ocnt, oagree, ostats = og.balance(T, seed, with_stats=True)
+    ocnt, oagree, ostats = og.balance(T, seed, with_stats=True, sampler=opts.get("sampler", 0))
     assert np.array_equal(cnt, ocnt), "edge flip counts"
     assert np.array_equal(agree, oagree), "vertex agree"
     assert list(ids) == list(range(T))
@@ -127,6 +127,42 @@ def test_harary_l224_procedure_on_gpu(which):
          "grid": lambda: graphgen.grid2d(40, 50, 0.5, 7)}[which]()
     st = check_cloud(g, 13, 2, harary=1, batch=5)
     assert st["harary_violations"] == 0
+
+
+def _uniform_graphs():
+    return {"er": graphgen.er(3000, 12000, 0.3, 4),
+            "chung_lu": graphgen.chung_lu(8000, 32000, 900, 0.75, 0.3, 5),
+            "forest": graphgen.er(4000, 2500, 0.4, 2),
+            "grid": graphgen.grid2d(30, 40, 0.5, 3),
+            "ring": graphgen.ring(300, neg_edges=(0, 7, 11))}
+
+
+@pytest.mark.parametrize("which", ["er", "chung_lu", "forest", "grid", "ring"])
+def test_uniform_sampler_trees_match_oracle(which):
+    """f.3 (Alg. 2 M = random, reading R17): the GPU's parallel cycle popping
+    returns exactly the oracle's sequential Wilson tree, and every later stage
+    (labels, walk, flips, cycle lengths) matches on it."""
+    g = _uniform_graphs()[which]
+    graphb.set_option("sampler", 1)
+    graphb.load_graph(g)
+    og = oracle.Graph.from_csr(g)
+    comp, coff, _ = og.components()
+    for t in range(4):
+        d = graphb.tree_debug(t, 9)
+        parent, _ = og.wilson_tree(9, t)
+        assert np.array_equal(d["parent"], parent), "uniform tree differs from the oracle's"
+        flip, sk, nc, _ = og.balance_tree(parent)
+        opre, osize = og.preorder(parent)
+        assert np.array_equal(d["size"], osize)
+        assert np.array_equal(d["flip"], flip)
+        assert d["sum_cycle_len"] == sk and d["num_cycles"] == nc
+        valid_preorder(d["parent"], d["size"], d["pre"], coff[comp])
+
+
+@pytest.mark.parametrize("which", ["er", "chung_lu", "forest"])
+def test_uniform_sampler_cloud(which):
+    """f.3: the frustration cloud over uniform spanning trees = the oracle's."""
+    check_cloud(_uniform_graphs()[which], 6, 4, sampler=1)
 
 
 def test_frustration_cloud_distinct_states():
