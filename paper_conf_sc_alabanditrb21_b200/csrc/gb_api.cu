@@ -55,6 +55,7 @@ struct Options {
     int64_t recpass = 1;     // walk 0: pre-indexed records scattered after the top-down pass
     int64_t persist = 0;     // bytes of L2 persisting window over the labelling arrays (0 = off)
     int64_t sampler = 0;     // Alg. 2 M: 0 BFS (R4), 1 uniform spanning trees (Wilson, R17)
+    int64_t wilson = 0;      // sampler 1: 0 one thread per tree (W trees at once), 1 parallel cycle popping
     int64_t harary = 0;      // 1: Harary sides by the L224 procedure (gb_harary.cu)
     int64_t jump = 1;        // walk 0: levels per ancestor record of the cycle walk (1, 2, 4)
 };
@@ -92,7 +93,7 @@ static void free_ws(Workspace &w) {
                     w.parq, w.offq, w.szq, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
                     w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof,
-                    w.jrec, w.hlab, w.wbuf, w.wparent};
+                    w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey};
     for (void *p : ptrs) if (p) cudaFree(p);
     w = Workspace();
 }
@@ -270,6 +271,11 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     std::vector<cudaEvent_t> evs;
     const bool timing = S.opt.timing != 0;
     int64_t done = 0;
+    // uniform sampler: trees per sampling chunk (<= kMaxBatch, ~2 GB of walk state)
+    const int64_t Wc = std::max<int64_t>(1, std::min<int64_t>({(int64_t)kMaxBatch, K,
+                                             (int64_t)(2.0e9 / (9.0 * (double)S.g.n))}));
+    cudaEvent_t wev[2];
+    double sample_ms = 0;
     while (done < K) {
         const int nb = (int)std::min<int64_t>(B, K - done);
         const int64_t t0 = t_begin + done * stride;
@@ -285,8 +291,33 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 3 * nb, st));
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
-        rc = run_batch_tree(S.g, S.ws, nb, nullptr, st, &T.launches, ev, descent, auto_sub(nb),
-                            (int)S.opt.recpass, (size_t)S.opt.persist, (int)S.opt.sampler);
+        const int32_t *given = nullptr;
+        if (S.opt.sampler == 1 && !S.opt.wilson) {
+            // uniform trees: sample the next chunk of W trees at once (one
+            // thread each), then label and walk them one by one
+            const int64_t j = done % Wc;
+            if (j == 0) {
+                const int W = (int)std::min<int64_t>(Wc, K - done);
+                if (!S.ws.wtkey) GB_CUDA_TRY(cudaMalloc(&S.ws.wtkey, sizeof(uint64_t) * kMaxBatch));
+                k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.wtkey, W, seed, t0, stride);
+                ++T.launches;
+                if (timing) { cudaEventCreate(&wev[0]); cudaEventCreate(&wev[1]); GB_CUDA_TRY(cudaEventRecord(wev[0], st)); }
+                rc = run_wilson_batch(S.g, S.ws, W, st, &T.launches);
+                if (rc) return rc;
+                if (timing) {
+                    GB_CUDA_TRY(cudaEventRecord(wev[1], st));
+                    GB_CUDA_TRY(cudaEventSynchronize(wev[1]));
+                    float ms = 0;
+                    cudaEventElapsedTime(&ms, wev[0], wev[1]);
+                    sample_ms += ms;
+                    cudaEventDestroy(wev[0]);
+                    cudaEventDestroy(wev[1]);
+                }
+            }
+            given = reinterpret_cast<const int32_t *>(S.ws.wseq) + j * S.g.n;
+        }
+        rc = run_batch_tree(S.g, S.ws, nb, given, st, &T.launches, ev, descent, auto_sub(nb),
+                            (int)S.opt.recpass, (size_t)S.opt.persist, given ? 0 : (int)S.opt.sampler);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
         rc = run_batch_cycles(S.g, S.ws, nb, G, descent, st, &T.launches, jump);
@@ -338,6 +369,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
             }
         }
         for (auto e : evs) cudaEventDestroy(e);
+        T.phase_ms[GB_PHASE_BFS] += sample_ms;
     }
     return GB_OK;
 }
@@ -353,10 +385,19 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 3, st));
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
+    const bool user_tree = d_given != nullptr;
+    if (!d_given && S.opt.sampler == 1 && !S.opt.wilson) {
+        if (!S.ws.wtkey) GB_CUDA_TRY(cudaMalloc(&S.ws.wtkey, sizeof(uint64_t) * kMaxBatch));
+        k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.wtkey, 1, seed, t, 1);
+        ++T.launches;
+        rc = run_wilson_batch(S.g, S.ws, 1, st, &T.launches);
+        if (rc) return rc;
+        d_given = reinterpret_cast<const int32_t *>(S.ws.wseq);
+    }
     rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk == 1, 1,
                         0, 0, d_given ? 0 : (int)S.opt.sampler);
     if (rc) return rc;
-    if (d_given) {
+    if (user_tree) {
         unsigned long long vis = 0;
         GB_CUDA_TRY(cudaMemcpyAsync(&vis, S.ws.visited, sizeof(vis), cudaMemcpyDeviceToHost, st));
         GB_CUDA_TRY(cudaStreamSynchronize(st));
@@ -514,6 +555,7 @@ int gb_set_option(const char *key, int64_t value) {
     else if (!strcmp(key, "msprof")) S.opt.msprof = value != 0;
     else if (!strcmp(key, "reset")) S.opt = Options();
     else if (!strcmp(key, "harary")) S.opt.harary = value != 0;
+    else if (!strcmp(key, "wilson")) S.opt.wilson = value != 0;
     else if (!strcmp(key, "sampler")) {
         if (value != 0 && value != 1) { set_error("sampler must be 0 (BFS) or 1 (uniform)"); return GB_EINVAL; }
         S.opt.sampler = value;

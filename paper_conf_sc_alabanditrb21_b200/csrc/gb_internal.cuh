@@ -156,7 +156,11 @@ struct Workspace {
     uint32_t *pp = nullptr;    // v: pre | pi<<31  (pi = root-path parity)
     uint2 *rec = nullptr;      // pre: {up pre | neg<<31, size}
     uint32_t *fbits = nullptr; // [B][ceil(m/32)] flip bitmask
-    void *wbuf = nullptr;      // option "sampler" = 1: Wilson state (20n bytes)
+    void *wbuf = nullptr;      // option "sampler" = 1, "wilson" = 1: cycle-popping state (20n bytes)
+    void *wseq = nullptr;      // option "sampler" = 1: [W] trees of per-thread Wilson state (9n bytes each);
+                               // the first 4Wn bytes are the W parent arrays
+    int wseq_cap = 0;
+    uint64_t *wtkey = nullptr; // [kMaxBatch] tree keys of the sampled chunk
     int32_t *wparent = nullptr;// its tree (parent, -1 at the roots)
     int32_t *hlab = nullptr;   // option "harary": [3n + 16] CC labels, CC roots, BFS levels, flag
     uint2 *jrec = nullptr;     // [G][n][K] K-level ancestor records of one cycle group (option "jump")
@@ -235,6 +239,9 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
 // cycle popping, gb_wilson.cu) -> parent (-1 at the roots)
 int run_wilson(const Graph &g, Workspace &ws, cudaStream_t st, int64_t *launches, int32_t *parent,
                int64_t *rounds_out);
+// f.3 default: W uniform spanning forests (keys ws.wtkey[0..W)), one GPU
+// thread per tree, into the first W*n int32 of ws.wseq
+int run_wilson_batch(const Graph &g, Workspace &ws, int W, cudaStream_t st, int64_t *launches);
 
 // multi-source BFS of the B <= kMsBatch sampled trees of a batch (roots, BFS
 // levels, min-hash parents); fills the level lists qv / parq, lvl, vbase, depth

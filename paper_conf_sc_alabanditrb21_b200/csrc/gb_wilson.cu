@@ -24,6 +24,8 @@
 #include "../../include/graphb.h"
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 
 namespace gb {
 
@@ -127,6 +129,70 @@ __global__ void k_w_parent(WParams P, int32_t *parent) {
         parent[u] = P.nxt[u] == (uint32_t)u ? -1 : (int32_t)P.nxt[u];
 }
 
+// ---------------------------------------------------------------------------
+// The default sampler: Wilson's algorithm exactly as the oracle runs it, one
+// GPU thread per tree (a batch of W trees at once).  The walks of one tree
+// are sequential (each loop-erased walk ends on the tree the previous ones
+// built), so the parallelism is across trees; per tree the state is a byte
+// (in tree), the stack depth and the last exit of every vertex.
+// ---------------------------------------------------------------------------
+struct WSeqParams {
+    const uint32_t *row_ptr, *adj;
+    const int32_t *coff, *cverts;
+    int64_t n, ncomp;
+    int W;
+    const uint64_t *tkey;    // [W]
+    uint8_t *in_tree;        // [W][n]
+    uint32_t *dep;           // [W][n]
+    int32_t *nxt;            // [W][n] -> parent (-1 at the roots)
+};
+
+__global__ void k_ws_init(WSeqParams P) {
+    const int64_t total = (int64_t)P.W * P.n;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        P.in_tree[i] = 0;
+        P.dep[i] = 0;
+        P.nxt[i] = -1;
+    }
+}
+
+__global__ void k_ws_roots(WSeqParams P) {
+    const int64_t total = (int64_t)P.W * P.ncomp;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const int b = (int)(i / P.ncomp);
+        const int64_t C = i - (int64_t)b * P.ncomp;
+        const uint32_t sz = (uint32_t)(P.coff[C + 1] - P.coff[C]);
+        const uint32_t r = (uint32_t)P.cverts[P.coff[C] + (int64_t)(root_key(P.tkey[b], C) % sz)];
+        P.in_tree[(size_t)b * P.n + r] = 1;
+    }
+}
+
+__global__ void k_ws_walks(WSeqParams P) {
+    const int b = blockIdx.x * blockDim.x + threadIdx.x;
+    if (b >= P.W) return;
+    const uint64_t tk = P.tkey[b];
+    uint8_t *in_tree = P.in_tree + (size_t)b * P.n;
+    uint32_t *dep = P.dep + (size_t)b * P.n;
+    int32_t *nxt = P.nxt + (size_t)b * P.n;
+    for (int64_t v = 0; v < P.n; v++) {
+        if (in_tree[v]) continue;
+        // random walk from v until it hits the tree; nxt keeps the last exit
+        uint32_t u = (uint32_t)v;
+        while (!in_tree[u]) {
+            const uint32_t rs = __ldg(P.row_ptr + u), deg = __ldg(P.row_ptr + u + 1) - rs;
+            const uint32_t j = dep[u]++;
+            const uint64_t h = mix64(tk + kWMul * (((uint64_t)u << 32) | j));
+            const uint32_t w = __ldg(P.adj + rs + (uint32_t)(h % deg)) & kIdMask;
+            nxt[u] = (int32_t)w;
+            u = w;
+        }
+        // the loop-erased path joins the tree
+        for (u = (uint32_t)v; !in_tree[u]; u = (uint32_t)nxt[u]) in_tree[u] = 1;
+    }
+}
+
 static unsigned wgrid(int64_t work, int sms) {
     return (unsigned)std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, (int64_t)sms * 8));
 }
@@ -155,6 +221,7 @@ int run_wilson(const Graph &g, Workspace &ws, cudaStream_t st, int64_t *launches
     k_w_roots<<<wgrid(g.ncomp, sms), 256, 0, st>>>(P);
     *launches += 2;
     int64_t active = n - g.ncomp, rounds = 0;
+    static const bool trace = getenv("GB_WILSON_TRACE") != nullptr;
     while (active > 0) {
         if (++rounds > (1 << 22)) { set_error("wilson: cycle popping did not finish"); return GB_ECUDA; }
         int K = 1;
@@ -175,10 +242,38 @@ int run_wilson(const Graph &g, Workspace &ws, cudaStream_t st, int64_t *launches
         GB_CUDA_TRY(cudaMemcpyAsync(&h, P.active, sizeof(h), cudaMemcpyDeviceToHost, st));
         GB_CUDA_TRY(cudaStreamSynchronize(st));
         active = (int64_t)h;
+        if (trace && (rounds < 64 || (rounds & (rounds - 1)) == 0 || active < 64))
+            fprintf(stderr, "wilson round %lld K %d active %lld\n", (long long)rounds, K, (long long)active);
     }
+    if (trace) fprintf(stderr, "wilson rounds %lld\n", (long long)rounds);
     k_w_parent<<<gn, 256, 0, st>>>(P, parent);
     ++*launches;
     if (rounds_out) *rounds_out = rounds;
+    GB_CUDA_TRY(cudaGetLastError());
+    return GB_OK;
+}
+
+int run_wilson_batch(const Graph &g, Workspace &ws, int W, cudaStream_t st, int64_t *launches) {
+    const int64_t n = g.n;
+    if (ws.wseq_cap < W) {
+        if (ws.wseq) cudaFree(ws.wseq);
+        ws.wseq = nullptr;
+        ws.wseq_cap = 0;
+        GB_CUDA_TRY(cudaMalloc(&ws.wseq, (size_t)W * 9 * (size_t)n + 64));
+        ws.wseq_cap = W;
+    }
+    WSeqParams P;
+    P.row_ptr = g.row_ptr; P.adj = g.adj; P.coff = g.coff; P.cverts = g.cverts;
+    P.n = n; P.ncomp = g.ncomp; P.W = W; P.tkey = ws.wtkey;
+    char *base = reinterpret_cast<char *>(ws.wseq);
+    P.nxt = reinterpret_cast<int32_t *>(base);
+    P.dep = reinterpret_cast<uint32_t *>(base + 4 * (size_t)W * n);
+    P.in_tree = reinterpret_cast<uint8_t *>(base + 8 * (size_t)W * n);
+    const int sms = g.num_sms;
+    k_ws_init<<<wgrid((int64_t)W * n, sms), 256, 0, st>>>(P);
+    k_ws_roots<<<wgrid((int64_t)W * g.ncomp, sms), 256, 0, st>>>(P);
+    k_ws_walks<<<(unsigned)W, 1, 0, st>>>(P);   // one tree per SM-resident thread
+    *launches += 3;
     GB_CUDA_TRY(cudaGetLastError());
     return GB_OK;
 }

@@ -137,13 +137,15 @@ def _uniform_graphs():
             "ring": graphgen.ring(300, neg_edges=(0, 7, 11))}
 
 
+@pytest.mark.parametrize("wilson", [0, 1])
 @pytest.mark.parametrize("which", ["er", "chung_lu", "forest", "grid", "ring"])
-def test_uniform_sampler_trees_match_oracle(which):
+def test_uniform_sampler_trees_match_oracle(which, wilson):
     """f.3 (Alg. 2 M = random, reading R17): the GPU's parallel cycle popping
     returns exactly the oracle's sequential Wilson tree, and every later stage
     (labels, walk, flips, cycle lengths) matches on it."""
     g = _uniform_graphs()[which]
     graphb.set_option("sampler", 1)
+    graphb.set_option("wilson", wilson)     # 0: thread per tree, 1: parallel cycle popping
     graphb.load_graph(g)
     og = oracle.Graph.from_csr(g)
     comp, coff, _ = og.components()
@@ -159,10 +161,12 @@ def test_uniform_sampler_trees_match_oracle(which):
         valid_preorder(d["parent"], d["size"], d["pre"], coff[comp])
 
 
+@pytest.mark.parametrize("wilson", [0, 1])
 @pytest.mark.parametrize("which", ["er", "chung_lu", "forest"])
-def test_uniform_sampler_cloud(which):
-    """f.3: the frustration cloud over uniform spanning trees = the oracle's."""
-    check_cloud(_uniform_graphs()[which], 6, 4, sampler=1)
+def test_uniform_sampler_cloud(which, wilson):
+    """f.3: the frustration cloud over uniform spanning trees = the oracle's
+    (several sampling chunks: T = 6 with at most 4 trees per chunk below)."""
+    check_cloud(_uniform_graphs()[which], 6, 4, sampler=1, wilson=wilson)
 
 
 def test_frustration_cloud_distinct_states():
