@@ -70,6 +70,8 @@ def lib():
         L.or_balance_m.restype = ctypes.c_int
         L.or_balance_m.argtypes = [P, i64, i64, i64, u64, ctypes.c_int, P, P, P]
         L.or_wdraw.restype = u64; L.or_wdraw.argtypes = [u64, i64, ctypes.c_int32, ctypes.c_uint32]
+        L.or_dfs_tree.restype = ctypes.c_int
+        L.or_dfs_tree.argtypes = [P, u64, i64, P]
         L.or_wilson_tree.restype = ctypes.c_int
         L.or_wilson_tree.argtypes = [P, u64, i64, ctypes.c_int, P, P]
         _lib = L
@@ -203,9 +205,17 @@ class Graph:
             raise OracleError(rc, "or_wilson_tree")
         return parent, pops
 
+    def dfs_tree(self, seed, t):
+        """Random-start DFS tree (reading R18): parent (-1 at the roots)."""
+        parent = np.zeros(self.n, np.int32)
+        rc = lib().or_dfs_tree(self._h, seed, t, _p(parent))
+        if rc != OR_OK:
+            raise OracleError(rc, "or_dfs_tree")
+        return parent
+
     def balance(self, num_trees, seed, t_begin=0, stride=1, with_stats=False, sampler=0):
         """Frustration cloud over trees t_begin, t_begin+stride, ... < num_trees
-        (sampler 0 = BFS trees, 1 = uniform spanning trees)."""
+        (sampler 0 = BFS trees, 1 = uniform spanning trees, 2 = DFS trees)."""
         cnt = np.zeros(max(self.m, 1), np.uint32); agree = np.zeros(self.n, np.uint32)
         k = len(range(t_begin, num_trees, stride))
         stats = np.zeros(4 * max(k, 1), np.uint64)

@@ -328,6 +328,49 @@ int or_wilson_tree(const or_graph *g, uint64_t seed, int64_t t, int order,
     return OR_OK;
 }
 
+/* ------------------------------------------------------------------------ */
+/* Tree sampling, Alg. 2 with M = DFS (L130), reading R18: a depth-first
+ * search from the R4 root of every component (components in rank order);
+ * at vertex u the neighbours are scanned from position
+ * dstart(u) = mix64(tkey ^ D*(u+1)) mod deg(u) cyclically, and the first
+ * unvisited one is descended into (returning to u resumes the scan).
+ * parent[w] = the vertex that discovered w.                                 */
+/* ------------------------------------------------------------------------ */
+#define OR_DMUL 0x8CB92BA72F3D8DD7ULL
+
+uint64_t or_dstart(uint64_t seed, int64_t t, int32_t u)
+{
+    return or_mix64(or_tkey(seed, t) ^ (OR_DMUL * ((uint64_t)(uint32_t)u + 1)));
+}
+
+int or_dfs_tree(const or_graph *g, uint64_t seed, int64_t t, int32_t *parent)
+{
+    int64_t n = g->n;
+    uint8_t *seen = (uint8_t *)calloc((size_t)n + 1, 1);
+    int64_t *pos = (int64_t *)calloc((size_t)n + 1, sizeof(int64_t));
+    int32_t *stack = (int32_t *)malloc(sizeof(int32_t) * ((size_t)n + 1));
+    if (!seen || !pos || !stack) { free(seen); free(pos); free(stack); return OR_ENOMEM; }
+    for (int64_t v = 0; v < n; v++) parent[v] = -1;
+    for (int64_t c = 0; c < g->ncomp; c++) {
+        int64_t sz = g->coff[c + 1] - g->coff[c];
+        int32_t r = g->cverts[g->coff[c] + (int64_t)(or_rkey(seed, t, c) % (uint64_t)sz)];
+        int64_t top = 0;
+        seen[r] = 1;
+        stack[top++] = r;
+        while (top > 0) {
+            int32_t u = stack[top - 1];
+            int64_t deg = g->row_ptr[u + 1] - g->row_ptr[u];
+            if (pos[u] == deg) { top--; continue; }
+            int64_t k = (int64_t)((or_dstart(seed, t, u) % (uint64_t)deg + (uint64_t)pos[u]) % (uint64_t)deg);
+            pos[u]++;
+            int32_t w = g->col[g->row_ptr[u] + k];
+            if (!seen[w]) { seen[w] = 1; parent[w] = u; stack[top++] = w; }
+        }
+    }
+    free(seen); free(pos); free(stack);
+    return OR_OK;
+}
+
 /* depth of every vertex under parent[], checking that parent[] is a spanning
  * forest of g with exactly one root per connected component. */
 static int tree_depth(const or_graph *g, const int32_t *parent, int32_t *depth, int8_t *pneg)
@@ -586,7 +629,7 @@ int or_balance(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride
     return or_balance_m(g, t_begin, t_end, stride, seed, 0, cnt, agree, stats);
 }
 
-/* sampler: 0 = BFS (R4), 1 = uniform (Wilson, R17) */
+/* sampler: 0 = BFS (R4), 1 = uniform (Wilson, R17), 2 = DFS (R18) */
 int or_balance_m(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride,
                  uint64_t seed, int sampler, uint32_t *cnt, uint32_t *agree, uint64_t *stats)
 {
@@ -602,6 +645,7 @@ int or_balance_m(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stri
     int64_t i = 0;
     for (int64_t t = t_begin; t < t_end; t += stride, i++) {
         rc = sampler == 1 ? or_wilson_tree(g, seed, t, 0, parent, NULL)
+           : sampler == 2 ? or_dfs_tree(g, seed, t, parent)
                           : or_bfs_tree(g, seed, t, parent, dist, NULL);
         if (rc != OR_OK) goto out;
         uint64_t sk = 0;

@@ -81,7 +81,13 @@ uint64_t or_wdraw(uint64_t seed, int64_t t, int32_t u, uint32_t j);
 int or_wilson_tree(const or_graph *g, uint64_t seed, int64_t t, int order,
                    int32_t *parent, uint32_t *pops);
 
-/* or_balance with the sampler chosen: 0 = BFS (R4), 1 = uniform (Wilson). */
+/* Alg. 2 with M = DFS (reading R18): scan of u's neighbours starts at
+ * or_dstart(seed,t,u) mod deg(u) and wraps around; parent[root] = -1. */
+uint64_t or_dstart(uint64_t seed, int64_t t, int32_t u);
+int or_dfs_tree(const or_graph *g, uint64_t seed, int64_t t, int32_t *parent);
+
+/* or_balance with the sampler chosen: 0 = BFS (R4), 1 = uniform (Wilson),
+ * 2 = DFS (R18). */
 int or_balance_m(const or_graph *g, int64_t t_begin, int64_t t_end, int64_t stride,
                  uint64_t seed, int sampler, uint32_t *cnt, uint32_t *agree, uint64_t *stats);
 

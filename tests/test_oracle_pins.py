@@ -588,3 +588,46 @@ def test_wilson_cloud_balances_every_tree():
         _check_tree_result(g, og, parent, flip, sk)
     cnt, agree, st = og.balance(4, 3, with_stats=True, sampler=1)
     assert int(st[:, 1].sum()) == 4 * (g.m - g.n + og.ncomp)
+
+
+# --------------------------------------------------------------------------
+# f.3: Alg. 2 with M = DFS (L130), reading R18.  Pins: the defining property
+# of an undirected DFS tree -- every non-tree edge joins an ancestor and a
+# descendant (no cross edges) -- plus closed shapes: DFS trees of complete
+# graphs and rings are Hamiltonian paths; roots follow R4.
+# --------------------------------------------------------------------------
+
+def _ancestors(parent, v):
+    out = set()
+    while parent[v] >= 0:
+        v = int(parent[v])
+        out.add(v)
+    return out
+
+
+@pytest.mark.parametrize("which", ["er", "chung_lu", "forest", "grid"])
+def test_dfs_tree_has_no_cross_edges(which):
+    g = {"er": lambda: graphgen.er(300, 1100, 0.3, 3),
+         "chung_lu": lambda: graphgen.chung_lu(400, 1600, 60, 0.75, 0.3, 2),
+         "forest": lambda: graphgen.er(400, 250, 0.4, 2),
+         "grid": lambda: graphgen.grid2d(9, 11, 0.5, 4)}[which]()
+    og = oracle.Graph.from_csr(g)
+    for t in range(4):
+        parent = og.dfs_tree(5, t)
+        _, dist, _ = og.bfs_tree(5, t)
+        assert np.array_equal(np.flatnonzero(parent < 0), np.flatnonzero(dist == 0))   # R4 roots
+        anc = [_ancestors(parent, v) for v in range(g.n)]
+        for u, v, _ in bf.edge_list(g):
+            assert u in anc[v] or v in anc[u], "cross edge: not a DFS tree"
+        for v in range(g.n):
+            if parent[v] >= 0:
+                assert (min(v, int(parent[v])), max(v, int(parent[v]))) in {(a, b) for a, b, _ in bf.edge_list(g)}
+
+
+@pytest.mark.parametrize("g", [graphgen.complete(9), graphgen.ring(17)])
+def test_dfs_tree_of_complete_and_ring_is_a_path(g):
+    og = oracle.Graph.from_csr(g)
+    for t in range(5):
+        parent = og.dfs_tree(2, t)
+        depth = [len(_ancestors(parent, v)) for v in range(g.n)]
+        assert sorted(depth) == list(range(g.n))          # one vertex per level: a path
