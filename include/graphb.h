@@ -110,7 +110,9 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
  * R4), 1 = uniform random spanning trees by Wilson's algorithm with
  * per-vertex random stacks (reading R17), sampled on the GPU by parallel
  * cycle popping and processed one tree at a time; gb_tree_debug then reports
- * that tree), "reset" (every option back to its default). */
+ * that tree; 2 = DFS trees with a hashed scan start per vertex, reading R18),
+ * "wilson" (sampler 1: 0 = one GPU thread per tree, 1 = parallel cycle
+ * popping), "reset" (every option back to its default). */
 int gb_set_option(const char *key, int64_t value);
 
 /* Statistics of the last gb_balance / gb_balance_range call:

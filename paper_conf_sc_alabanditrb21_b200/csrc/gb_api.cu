@@ -207,7 +207,7 @@ __global__ void k_record_stats(const unsigned long long *tstat, const int32_t *d
 }
 
 static int auto_batch(int64_t ntrees) {
-    if (S.opt.sampler == 1) return 1;   // sampled trees go one at a time (caller-tree path)
+    if (S.opt.sampler != 0) return 1;   // sampled trees go one at a time (caller-tree path)
     if (S.opt.batch > 0) return (int)std::min<int64_t>(S.opt.batch, kMaxBatch);
     const size_t have = S.free_at_load;
     int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk == 1));
@@ -273,7 +273,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     int64_t done = 0;
     // uniform sampler: trees per sampling chunk (<= kMaxBatch, ~2 GB of walk state)
     const int64_t Wc = std::max<int64_t>(1, std::min<int64_t>({(int64_t)kMaxBatch, K,
-                                             (int64_t)(2.0e9 / (9.0 * (double)S.g.n))}));
+                                             (int64_t)(2.0e9 / (13.0 * (double)S.g.n))}));
     cudaEvent_t wev[2];
     double sample_ms = 0;
     while (done < K) {
@@ -292,7 +292,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
         const int32_t *given = nullptr;
-        if (S.opt.sampler == 1 && !S.opt.wilson) {
+        if (S.opt.sampler == 2 || (S.opt.sampler == 1 && !S.opt.wilson)) {
             // uniform trees: sample the next chunk of W trees at once (one
             // thread each), then label and walk them one by one
             const int64_t j = done % Wc;
@@ -302,7 +302,8 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
                 k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.wtkey, W, seed, t0, stride);
                 ++T.launches;
                 if (timing) { cudaEventCreate(&wev[0]); cudaEventCreate(&wev[1]); GB_CUDA_TRY(cudaEventRecord(wev[0], st)); }
-                rc = run_wilson_batch(S.g, S.ws, W, st, &T.launches);
+                rc = S.opt.sampler == 2 ? run_dfs_batch(S.g, S.ws, W, st, &T.launches)
+                                        : run_wilson_batch(S.g, S.ws, W, st, &T.launches);
                 if (rc) return rc;
                 if (timing) {
                     GB_CUDA_TRY(cudaEventRecord(wev[1], st));
@@ -386,11 +387,12 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
     const bool user_tree = d_given != nullptr;
-    if (!d_given && S.opt.sampler == 1 && !S.opt.wilson) {
+    if (!d_given && (S.opt.sampler == 2 || (S.opt.sampler == 1 && !S.opt.wilson))) {
         if (!S.ws.wtkey) GB_CUDA_TRY(cudaMalloc(&S.ws.wtkey, sizeof(uint64_t) * kMaxBatch));
         k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.wtkey, 1, seed, t, 1);
         ++T.launches;
-        rc = run_wilson_batch(S.g, S.ws, 1, st, &T.launches);
+        rc = S.opt.sampler == 2 ? run_dfs_batch(S.g, S.ws, 1, st, &T.launches)
+                                : run_wilson_batch(S.g, S.ws, 1, st, &T.launches);
         if (rc) return rc;
         d_given = reinterpret_cast<const int32_t *>(S.ws.wseq);
     }
@@ -557,7 +559,7 @@ int gb_set_option(const char *key, int64_t value) {
     else if (!strcmp(key, "harary")) S.opt.harary = value != 0;
     else if (!strcmp(key, "wilson")) S.opt.wilson = value != 0;
     else if (!strcmp(key, "sampler")) {
-        if (value != 0 && value != 1) { set_error("sampler must be 0 (BFS) or 1 (uniform)"); return GB_EINVAL; }
+        if (value < 0 || value > 2) { set_error("sampler must be 0 (BFS), 1 (uniform) or 2 (DFS)"); return GB_EINVAL; }
         S.opt.sampler = value;
     }
     else if (!strcmp(key, "recpass")) S.opt.recpass = value != 0;

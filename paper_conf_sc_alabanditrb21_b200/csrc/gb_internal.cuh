@@ -157,7 +157,7 @@ struct Workspace {
     uint2 *rec = nullptr;      // pre: {up pre | neg<<31, size}
     uint32_t *fbits = nullptr; // [B][ceil(m/32)] flip bitmask
     void *wbuf = nullptr;      // option "sampler" = 1, "wilson" = 1: cycle-popping state (20n bytes)
-    void *wseq = nullptr;      // option "sampler" = 1: [W] trees of per-thread Wilson state (9n bytes each);
+    void *wseq = nullptr;      // option "sampler" = 1, 2: [W] trees of per-thread sampler state (13n bytes each);
                                // the first 4Wn bytes are the W parent arrays
     int wseq_cap = 0;
     uint64_t *wtkey = nullptr; // [kMaxBatch] tree keys of the sampled chunk
@@ -242,6 +242,8 @@ int run_wilson(const Graph &g, Workspace &ws, cudaStream_t st, int64_t *launches
 // f.3 default: W uniform spanning forests (keys ws.wtkey[0..W)), one GPU
 // thread per tree, into the first W*n int32 of ws.wseq
 int run_wilson_batch(const Graph &g, Workspace &ws, int W, cudaStream_t st, int64_t *launches);
+// f.3: W DFS trees (reading R18), one GPU thread per tree, same output place
+int run_dfs_batch(const Graph &g, Workspace &ws, int W, cudaStream_t st, int64_t *launches);
 
 // multi-source BFS of the B <= kMsBatch sampled trees of a batch (roots, BFS
 // levels, min-hash parents); fills the level lists qv / parq, lvl, vbase, depth

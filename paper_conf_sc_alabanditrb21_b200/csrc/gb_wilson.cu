@@ -253,15 +253,101 @@ int run_wilson(const Graph &g, Workspace &ws, cudaStream_t st, int64_t *launches
     return GB_OK;
 }
 
-int run_wilson_batch(const Graph &g, Workspace &ws, int W, cudaStream_t st, int64_t *launches) {
-    const int64_t n = g.n;
+// ---------------------------------------------------------------------------
+// Alg. 2 with M = DFS (reading R18), one GPU thread per tree: iterative DFS
+// from the R4 root of every component; the scan of u's neighbours starts at
+// mix64(tkey ^ D*(u+1)) mod deg(u) and wraps around.
+// ---------------------------------------------------------------------------
+constexpr uint64_t kDMul = 0x8CB92BA72F3D8DD7ull;
+
+struct DfsParams {
+    const uint32_t *row_ptr, *adj;
+    const int32_t *coff, *cverts;
+    int64_t n, ncomp;
+    int W;
+    const uint64_t *tkey;    // [W]
+    int32_t *parent;         // [W][n]
+    uint32_t *pos;           // [W][n] neighbours scanned so far
+    uint8_t *seen;           // [W][n]
+    uint32_t *stack;         // [W][n]
+};
+
+__global__ void k_ds_init(DfsParams P) {
+    const int64_t total = (int64_t)P.W * P.n;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        P.parent[i] = -1;
+        P.pos[i] = 0;
+        P.seen[i] = 0;
+    }
+}
+
+__global__ void k_ds_dfs(DfsParams P) {
+    const int b = blockIdx.x * blockDim.x + threadIdx.x;
+    if (b >= P.W) return;
+    const uint64_t tk = P.tkey[b];
+    const size_t o = (size_t)b * P.n;
+    int32_t *parent = P.parent + o;
+    uint32_t *pos = P.pos + o, *stack = P.stack + o;
+    uint8_t *seen = P.seen + o;
+    for (int64_t C = 0; C < P.ncomp; C++) {
+        const uint32_t sz = (uint32_t)(P.coff[C + 1] - P.coff[C]);
+        const uint32_t r = (uint32_t)P.cverts[P.coff[C] + (int64_t)(root_key(tk, C) % sz)];
+        int64_t top = 0;
+        seen[r] = 1;
+        stack[top++] = r;
+        while (top > 0) {
+            const uint32_t u = stack[top - 1];
+            const uint32_t rs = __ldg(P.row_ptr + u), deg = __ldg(P.row_ptr + u + 1) - rs;
+            const uint32_t p = pos[u];
+            if (p == deg) { top--; continue; }
+            const uint32_t s0 = (uint32_t)(mix64(tk ^ (kDMul * ((uint64_t)u + 1))) % deg);
+            const uint32_t k = s0 + p >= deg ? s0 + p - deg : s0 + p;
+            pos[u] = p + 1;
+            const uint32_t w = __ldg(P.adj + rs + k) & kIdMask;
+            if (!seen[w]) {
+                seen[w] = 1;
+                parent[w] = (int32_t)u;
+                stack[top++] = w;
+            }
+        }
+    }
+}
+
+static int ensure_sampler_state(const Graph &g, Workspace &ws, int W) {
     if (ws.wseq_cap < W) {
         if (ws.wseq) cudaFree(ws.wseq);
         ws.wseq = nullptr;
         ws.wseq_cap = 0;
-        GB_CUDA_TRY(cudaMalloc(&ws.wseq, (size_t)W * 9 * (size_t)n + 64));
+        GB_CUDA_TRY(cudaMalloc(&ws.wseq, (size_t)W * 13 * (size_t)g.n + 64));
         ws.wseq_cap = W;
     }
+    return GB_OK;
+}
+
+int run_dfs_batch(const Graph &g, Workspace &ws, int W, cudaStream_t st, int64_t *launches) {
+    const int64_t n = g.n;
+    int rc = ensure_sampler_state(g, ws, W);
+    if (rc) return rc;
+    DfsParams P;
+    P.row_ptr = g.row_ptr; P.adj = g.adj; P.coff = g.coff; P.cverts = g.cverts;
+    P.n = n; P.ncomp = g.ncomp; P.W = W; P.tkey = ws.wtkey;
+    char *base = reinterpret_cast<char *>(ws.wseq);
+    P.parent = reinterpret_cast<int32_t *>(base);
+    P.pos = reinterpret_cast<uint32_t *>(base + 4 * (size_t)W * n);
+    P.seen = reinterpret_cast<uint8_t *>(base + 8 * (size_t)W * n);
+    P.stack = reinterpret_cast<uint32_t *>(base + ((9 * (size_t)W * n + 15) & ~(size_t)15));
+    k_ds_init<<<wgrid((int64_t)W * n, g.num_sms), 256, 0, st>>>(P);
+    k_ds_dfs<<<(unsigned)W, 1, 0, st>>>(P);
+    *launches += 2;
+    GB_CUDA_TRY(cudaGetLastError());
+    return GB_OK;
+}
+
+int run_wilson_batch(const Graph &g, Workspace &ws, int W, cudaStream_t st, int64_t *launches) {
+    const int64_t n = g.n;
+    int rc0 = ensure_sampler_state(g, ws, W);
+    if (rc0) return rc0;
     WSeqParams P;
     P.row_ptr = g.row_ptr; P.adj = g.adj; P.coff = g.coff; P.cverts = g.cverts;
     P.n = n; P.ncomp = g.ncomp; P.W = W; P.tkey = ws.wtkey;

@@ -169,6 +169,33 @@ def test_uniform_sampler_cloud(which, wilson):
     check_cloud(_uniform_graphs()[which], 6, 4, sampler=1, wilson=wilson)
 
 
+@pytest.mark.parametrize("which", ["er", "chung_lu", "forest", "grid", "ring"])
+def test_dfs_sampler_trees_match_oracle(which):
+    """f.3 (Alg. 2 M = DFS, reading R18): the GPU's DFS tree equals the
+    oracle's, and labels / walk / flips / cycle lengths match on it."""
+    g = _uniform_graphs()[which]
+    graphb.set_option("sampler", 2)
+    graphb.load_graph(g)
+    og = oracle.Graph.from_csr(g)
+    comp, coff, _ = og.components()
+    for t in range(3):
+        d = graphb.tree_debug(t, 5)
+        parent = og.dfs_tree(5, t)
+        assert np.array_equal(d["parent"], parent), "DFS tree differs from the oracle's"
+        flip, sk, nc, _ = og.balance_tree(parent)
+        opre, osize = og.preorder(parent)
+        assert np.array_equal(d["size"], osize)
+        assert np.array_equal(d["flip"], flip)
+        assert d["sum_cycle_len"] == sk and d["num_cycles"] == nc
+        valid_preorder(d["parent"], d["size"], d["pre"], coff[comp])
+
+
+@pytest.mark.parametrize("which", ["er", "forest"])
+def test_dfs_sampler_cloud(which):
+    """f.3: the frustration cloud over DFS trees = the oracle's."""
+    check_cloud(_uniform_graphs()[which], 5, 6, sampler=2)
+
+
 def test_frustration_cloud_distinct_states():
     """f.2 (Fig. 2, L81/L86): distinct nearest balanced states over many
     trees, counted from the per-tree state signatures, equal the oracle's."""
