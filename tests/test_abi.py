@@ -59,6 +59,16 @@ def test_state_and_argument_errors_without_gpu():
     assert L.gb_load_csr(2, 1, rp.ctypes.data, None, None) == graphb.GB_EINVAL
     assert L.gb_set_option(b"nope", 1) == graphb.GB_EINVAL
     assert L.gb_set_option(b"walk", 2) == graphb.GB_EINVAL
+    assert L.gb_set_option(b"sampler", 3) == graphb.GB_EINVAL      # BFS, uniform, DFS only
+    assert L.gb_set_option(b"sampler", -1) == graphb.GB_EINVAL
+    assert L.gb_set_option(b"jump", 3) == graphb.GB_EINVAL         # 1, 2 or 4 levels
+    for k, v in [(b"sampler", 2), (b"wilson", 1), (b"harary", 1), (b"jump", 4), (b"recpass", 0)]:
+        assert L.gb_set_option(k, v) == 0
+    assert L.gb_set_option(b"reset", 0) == 0
+    # label / BFS profiles need the msprof option (and a run)
+    buf = np.zeros(1024, np.uint64)
+    assert L.gb_label_profile(buf.ctypes.data) == graphb.GB_ESTATE
+    assert L.gb_msbfs_profile(buf.ctypes.data) == graphb.GB_ESTATE
 
 
 @pytest.mark.skipif(__import__("tests.conftest", fromlist=["x"]).cuda_available(),
