@@ -343,7 +343,13 @@ def main():
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(g, 1, sample_trees_for(g, args.cpu_sample_trees), c_nt)
+        if g.m > 2e8 and not args.cpu_sample_trees:
+            # the single-threaded oracle needs minutes just to build a 1 B-edge graph
+            cpu = {"value": None, "unit": "cycles/s", "cores": 1, "kind": "oracle",
+                   "sample": "not run: m > 2e8 exceeds the bounded-sample budget "
+                             "(pass --cpu-sample-trees 1 to force one tree)"}
+        else:
+            cpu = cpu_baseline(g, 1, sample_trees_for(g, args.cpu_sample_trees), c_nt)
 
     if rank == 0:
         line = {
