@@ -326,12 +326,21 @@ def main():
             dist.barrier()
         torch.cuda.synchronize()
         t0 = time.perf_counter()
+        trace = os.environ.get("GB_E2E_TRACE")
         for s in range(e_steps):
+            ta = time.perf_counter()
             graphb.load_csr(hrp, hcol, hsg)
+            tb = time.perf_counter()
             cnt.zero_(); agree.zero_()
             step(500 + s)
+            if trace:
+                torch.cuda.synchronize()
+            tc = time.perf_counter()
             h_cnt.copy_(cnt); h_agr.copy_(agree)
             torch.cuda.synchronize()
+            if trace:
+                print(f"e2e step {s}: load {1e3 * (tb - ta):.1f} ms, balance {1e3 * (tc - tb):.1f} ms, "
+                      f"d2h {1e3 * (time.perf_counter() - tc):.1f} ms", file=sys.stderr, flush=True)
         el = time.perf_counter() - t0
         tt = torch.tensor([el], dtype=torch.float64, device=dev)
         if world > 1:

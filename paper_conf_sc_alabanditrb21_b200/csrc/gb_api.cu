@@ -507,9 +507,10 @@ int gb_load_csr(int64_t n, int64_t m, const int64_t *row_ptr, const int32_t *col
     int64_t launches = 0;
     rc = ingest(S.g, n, m, row_ptr, col_idx, sign, S.stream, &launches);
     if (rc) { gb_free(); return rc; }
-    if (S.ws.B && (S.g.n != old_n || S.g.m != old_m || S.g.ncomp != old_c || S.g.nmulti != old_h))
-        free_ws(S.ws);
-    {
+    const bool same_shape = S.g.n == old_n && S.g.m == old_m && S.g.ncomp == old_c && S.g.nmulti == old_h;
+    if (S.ws.B && !same_shape) free_ws(S.ws);
+    if (!same_shape || !S.ws.B || !S.free_at_load) {
+        // a same-shape reload keeps the workspace and the memory estimate
         size_t freeb = 0, totb = 0;
         GB_CUDA_TRY(cudaMemGetInfo(&freeb, &totb));
         S.free_at_load = freeb + (size_t)S.ws.B * per_tree_bytes(S.g, S.ws_descent);

@@ -402,6 +402,14 @@ __device__ __forceinline__ void load_level(const TreeParams &P, int L, LevelTabl
     __syncthreads();
 }
 
+// independent vertices per thread in the level passes (measured: 4)
+#ifndef GB_ILP_UP
+#define GB_ILP_UP 4
+#endif
+#ifndef GB_ILP_DOWN
+#define GB_ILP_DOWN 4
+#endif
+
 // Levels with at most kSolo vertices (the first and last levels of a BFS
 // tree) are processed by block 0 alone: consecutive small levels are
 // separated by __syncthreads instead of grid barriers, and the other blocks
@@ -520,7 +528,7 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
         if constexpr (!kDescent) {
             // kILP independent vertices per thread: their queue words, their
             // own sizes and the adds to their parents are in flight together
-            constexpr int kILP = 4;
+            constexpr int kILP = GB_ILP_UP;
             GB_QPOL;
             for (unsigned long long base = gtid; base < total; base += kILP * nthr) {
                 size_t qi[kILP], nbk[kILP];
@@ -630,7 +638,7 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
         if (!kDescent && L > 0) {
             // kILP independent vertices per thread per iteration: their queue
             // words, then their parents' labels, are in flight together
-            constexpr int kILP = 4;
+            constexpr int kILP = GB_ILP_DOWN;
             GB_QPOL;
             for (unsigned long long base = gtid; base < total; base += kILP * nthr) {
                 size_t qi[kILP], nbk[kILP];

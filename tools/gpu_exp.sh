@@ -1,5 +1,4 @@
-timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -2
-run() { timeout 300 python bench.py --config $CFG --no-cpu-baseline --no-e2e --steps 3 "$@" 2>&1 | tail -1 | python -c "
-import json,sys; d=json.loads(sys.stdin.read()); print('$LBL $CFG $*', round(d['value']/1e9,3), round(d['ms_per_step'],1), {k:round(v,1) for k,v in d['phase_ms_per_step'].items()})" ; }
-for CFG in c3 c2 c4; do run; done
-python tools/msprof.py c3 64 | tail -18
+run() { timeout 300 python bench.py --config c3 --no-cpu-baseline --no-e2e --steps 3 "$@" 2>&1 | tail -1 | python -c "
+import json,sys; d=json.loads(sys.stdin.read()); print('$LBL', round(d['value']/1e9,3), round(d['ms_per_step'],1), {k:round(v,1) for k,v in d['phase_ms_per_step'].items()})" ; }
+LBL=ilp4 run
+for v in v1 v2 v3; do LBL=$v GRAPHB_LIB=$PWD/paper_conf_sc_alabanditrb21_b200/libgraphb_$v.so run; done
