@@ -137,9 +137,9 @@ static int ensure_workspace(int B, bool descent) {
     ALLOC(w.fr, 2 * n);
     ALLOC(w.hacc, std::max<int64_t>(g.nmulti, 1));
     ALLOC(w.hbest, std::max<int64_t>(g.nmulti, 1) * kMsBatch);
-    ALLOC(w.msflag, 2);
+    ALLOC(w.msflag, 8);
     ALLOC(w.mscnt, (int64_t)kMsBatch * 2048);
-    ALLOC(w.fbm, 4 * ((n + 31) / 32));
+    ALLOC(w.fbm, 6 * ((n + 31) / 32));
     ALLOC(w.qv, Bn);
     ALLOC(w.lvl, (int64_t)B * (n + 2));
     ALLOC(w.vbase, (int64_t)B * (n + 2));

@@ -170,10 +170,12 @@ struct Workspace {
     unsigned long long *fr = nullptr;   // [2][n] frontier of level L / L+1
     unsigned long long *hacc = nullptr; // [nmulti] discoveries of multi-chunk vertices
     unsigned long long *hbest = nullptr;// [nmulti][64] their best parent keys
-    int32_t *msflag = nullptr;          // [2] a multi-chunk vertex discovered something
+    int32_t *msflag = nullptr;          // [8]: [0..1] a multi-chunk vertex discovered something,
+                                        // [4..6] frontier sizes (levels mod 3)
     uint32_t *mscnt = nullptr;          // [64][2048] per-block discovery counts
     unsigned long long *msprof = nullptr;  // [256][4] BFS phase timestamps (option "msprof")
-    uint32_t *fbm = nullptr;            // [4][ceil(n/32)] frontier bitmaps (3) + finished bitmap
+    uint32_t *fbm = nullptr;            // [6][ceil(n/32)] frontier bitmaps (3), finished bitmap,
+                                        // two push bitmaps (direction optimisation)
     uint32_t *s1 = nullptr;    // [B][ncomp] #vertices with pi = 1 per component
     uint64_t *tkey = nullptr;  // [kMaxBatch]
     int32_t *depth = nullptr;  // [kMaxBatch]

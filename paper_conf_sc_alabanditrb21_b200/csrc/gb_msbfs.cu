@@ -49,6 +49,9 @@ struct MsParams {
     unsigned long long *vis, *fr, *hacc, *hbest;
     uint32_t *fbm;     // [3][nwords] frontier bitmaps (level L % 3)
     uint32_t *fullbm;  // [nwords] finished vertices
+    uint32_t *tb;      // [2][nwords] "has a neighbour on the frontier" (push levels)
+    uint32_t *fcnt;    // [3] vertices on the frontier of level L (mod 3); [3] vertices finished
+    int64_t push_div;  // a level pushes first while frontier * push_div <= unfinished vertices
     int32_t *flag;
     uint32_t *mscnt;   // [64][kMsMaxBlocks] discoveries per tree per block (phase A)
     const uint64_t *tkey;
@@ -437,6 +440,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
     const int64_t ntiles = nit_tiles + nl_tiles;
     const unsigned long long full = P.full;
     const uint32_t nblk = gridDim.x;
+    __shared__ uint32_t s_fc, s_ff;
     for (int L = 0;; L++) {
         const unsigned long long *F = P.fr + (size_t)(L & 1) * P.n;
         unsigned long long *Nx = P.fr + (size_t)((L + 1) & 1) * P.n;
@@ -451,7 +455,42 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
         }
         // words written with atomics next level (items, the boundary word)
         for (int64_t w = gtid; w < P.itemwords; w += nthr) cbm[w] = 0;
+        if (tid == 0) { s_fc = 0; s_ff = 0; }
+        if (blockIdx.x == 0 && tid == 0) P.fcnt[(L + 2) % 3] = 0;
         __syncthreads();
+        // Direction optimisation: while the frontier is small (the first
+        // levels), push from it first -- every frontier vertex marks its
+        // neighbours in tbc -- so that the pull below reads the adjacency of
+        // marked vertices only (nothing else can be discovered).  Heavy
+        // vertices push through their work items (<= 256 slots per warp).
+        const uint32_t fc = L == 0 ? (uint32_t)(((int64_t)B * P.ncomp < P.n) ? (int64_t)B * P.ncomp : P.n)
+                                   : __ldcg(P.fcnt + L % 3);
+        const int64_t unfinished = P.n - (int64_t)__ldcg(P.fcnt + 3);
+        const bool push = (int64_t)fc * P.push_div <= unfinished;
+        uint32_t *tbc = P.tb + (size_t)(L & 1) * P.nwords;
+        if (push) {
+            for (int64_t k = gwarp; k < P.nitems; k += nwarps) {
+                const uint2 it = __ldg(P.items + k);
+                if (!bm_test(bm, it.x)) continue;
+                const uint32_t s1 = min(it.y + (uint32_t)kChunk, __ldg(P.brow + it.x + 1));
+                for (uint32_t j = it.y + lane; j < s1; j += 32) {
+                    const uint32_t x = __ldg(P.badj + j) & kIdMask;
+                    atomicOr(tbc + (x >> 5), 1u << (x & 31));
+                }
+            }
+            for (int64_t w = (P.nlight0 >> 5) + gwarp; w < P.nwords; w += nwarps) {
+                uint32_t word = __ldcg(bm + w);
+                if ((w << 5) < P.nlight0) word &= ~0u << (uint32_t)(P.nlight0 - (w << 5));   // item vertices done above
+                if (!((word >> lane) & 1u)) continue;
+                const uint32_t u = (uint32_t)(w * 32 + lane);
+                const uint32_t rs = __ldg(P.brow + u), re = __ldg(P.brow + u + 1);
+                for (uint32_t j = rs; j < re; j++) {
+                    const uint32_t x = __ldg(P.badj + j) & kIdMask;
+                    atomicOr(tbc + (x >> 5), 1u << (x & 31));
+                }
+            }
+            grid.sync();
+        }
         MS_PROF(0);
         // ---------------- phase A: discoveries --------------------------------
         for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
@@ -461,6 +500,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                     const uint2 it = __ldg(P.items + k);
                     const uint32_t i = it.x, s0 = it.y;
                     if (bm_test(P.fullbm, i)) continue;
+                    if (push && !bm_test(tbc, i)) continue;
                     const uint32_t s1 = min(s0 + (uint32_t)kChunk, __ldg(P.brow + i + 1));
                     const bool multi = k < P.nmulti_items;
                     const unsigned long long vis = __ldcg(P.vis + i);
@@ -475,10 +515,14 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                             Nx[i] = part;
                             P.vis[i] = vis | part;
                             atomicOr(nbm + (i >> 5), 1u << (i & 31));
-                            if ((vis | part) == full) atomicOr(P.fullbm + (i >> 5), 1u << (i & 31));
+                            if ((vis | part) == full) {
+                                atomicOr(P.fullbm + (i >> 5), 1u << (i & 31));
+                                atomicAdd(&s_ff, 1u);
+                            }
                         }
                         if ((part >> lane) & 1ull) atomicAdd(&s_cnt[lane], 1u);
                         if ((part >> (lane + 32)) & 1ull) atomicAdd(&s_cnt[lane + 32], 1u);
+                        if (lane == 0) atomicAdd(&s_fc, 1u);
                     }
                 }
             } else {
@@ -487,9 +531,10 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                 const uint32_t i = (uint32_t)(v0 + lane);
                 const bool mine = (int64_t)i < P.n && (int64_t)i >= P.nlight0;
                 const uint32_t fw = __ldcg(P.fullbm + (v0 >> 5));
+                const uint32_t tw = push ? __ldcg(tbc + (v0 >> 5)) : ~0u;
                 unsigned long long nw = 0;
                 bool nowfull = false;
-                if (mine && !((fw >> lane) & 1u)) {
+                if (mine && !((fw >> lane) & 1u) && ((tw >> lane) & 1u)) {
                     const unsigned long long vis = __ldcg(P.vis + i);
                     const uint32_t rs = __ldg(P.brow + i);
                     const uint32_t deg = __ldg(P.brow + i + 1) - rs;
@@ -510,6 +555,8 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                 }
                 const uint32_t fb = __ballot_sync(0xFFFFFFFFu, nw != 0);
                 const uint32_t nf = __ballot_sync(0xFFFFFFFFu, nowfull);
+                if (lane == 0 && fb) atomicAdd(&s_fc, (uint32_t)__popc(fb));
+                if (lane == 0 && nf) atomicAdd(&s_ff, (uint32_t)__popc(nf));
                 if (lane == 0) {
                     if (v0 >= P.nlight0) {
                         nbm[v0 >> 5] = fb;
@@ -526,6 +573,8 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
             P.mscnt[(size_t)tid * kMsMaxBlocks + blockIdx.x] = s_cnt[tid];
             s_cnt[tid] = 0;
         }
+        if (tid == 0 && s_fc) atomicAdd(P.fcnt + (L + 1) % 3, s_fc);
+        if (tid == 0 && s_ff) atomicAdd(P.fcnt + 3, s_ff);
         grid.sync();
         MS_PROF(1);
         // ---------------- phase B: parents ------------------------------------
@@ -598,6 +647,8 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
         __syncwarp();
         if (qn) ms_light_parents(P, F, Nx, bm, s_q[wid][lane], lane < qn, s_tk, s_base, s_pos, W);
         qn = 0;
+        // the push bitmap of level L + 1 starts empty
+        for (int64_t w = gtid; w < P.nwords; w += nthr) P.tb[(size_t)((L + 1) & 1) * P.nwords + w] = 0;
         // hubs: partial minima of every chunk
         const bool multi = P.nmulti_items > 0 && *(volatile int32_t *)(P.flag + (L & 1)) != 0;
         if (multi) {
@@ -636,12 +687,16 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                 }
                 __syncwarp();
                 if (lane == 0) {
+                    atomicAdd(P.fcnt + (L + 1) % 3, 1u);
                     const unsigned long long vis = __ldcg(P.vis + hi) | want;
                     P.vis[hi] = vis;
                     Nx[hi] = want;
                     P.hacc[hi] = 0;
                     atomicOr(nbm + (hi >> 5), 1u << (hi & 31));
-                    if (vis == full) atomicOr(P.fullbm + (hi >> 5), 1u << (hi & 31));
+                    if (vis == full) {
+                        atomicOr(P.fullbm + (hi >> 5), 1u << (hi & 31));
+                        atomicAdd(P.fcnt + 3, 1u);
+                    }
                 }
             }
             grid.sync();
@@ -692,14 +747,17 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
     P.full = B == 64 ? ~0ull : ((1ull << B) - 1);
     P.vis = ws.vis; P.fr = ws.fr; P.hacc = ws.hacc; P.hbest = ws.hbest;
     P.fbm = ws.fbm; P.fullbm = ws.fbm + 3 * P.nwords;
+    P.tb = ws.fbm + 4 * P.nwords;
+    P.fcnt = reinterpret_cast<uint32_t *>(ws.msflag + 4);
+    P.push_div = 32;   // measured on C3: 32 and 128 equal (bfs 59.0 ms / 100 trees), 8 worse (61.3)
     P.flag = ws.msflag; P.mscnt = ws.mscnt;
     P.tkey = o.tkey; P.qv = o.qv; P.parq = o.parq; P.pp = o.pp; P.rec = o.rec; P.crec = o.crec;
     P.lvl = o.lvl; P.vbase = o.vbase; P.depth = o.depth; P.maxd = o.maxd;
     P.prof = ws.msprof;
     GB_CUDA_TRY(cudaMemsetAsync(ws.vis, 0, sizeof(unsigned long long) * (size_t)g.n, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.fr, 0, sizeof(unsigned long long) * (size_t)g.n, st));
-    GB_CUDA_TRY(cudaMemsetAsync(ws.fbm, 0, sizeof(uint32_t) * 4 * (size_t)P.nwords, st));
-    GB_CUDA_TRY(cudaMemsetAsync(ws.msflag, 0, sizeof(int32_t) * 2, st));
+    GB_CUDA_TRY(cudaMemsetAsync(ws.fbm, 0, sizeof(uint32_t) * 6 * (size_t)P.nwords, st));
+    GB_CUDA_TRY(cudaMemsetAsync(ws.msflag, 0, sizeof(int32_t) * 8, st));
     const int64_t work = (int64_t)B * g.ncomp;
     k_ms_roots<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, 8192)), 256, 0, st>>>(P);
     ++*launches;
