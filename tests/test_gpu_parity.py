@@ -196,6 +196,16 @@ def test_dfs_sampler_cloud(which):
     check_cloud(_uniform_graphs()[which], 5, 6, sampler=2)
 
 
+@pytest.mark.parametrize("sampler,walk,harary", [(1, 1, 0), (2, 1, 0), (1, 0, 1), (2, 0, 1)])
+def test_samplers_with_descent_walk_and_l224_sides(sampler, walk, harary):
+    """f.3 samplers combined with Alg. 3's descent walk (walk 1) and with the
+    paper's L224 Harary procedure (f.2): still the oracle's cloud."""
+    g = graphgen.chung_lu(6000, 24000, 700, 0.75, 0.35, 12)
+    st = check_cloud(g, 5, 8, sampler=sampler, walk=walk, harary=harary)
+    if harary:
+        assert st["harary_violations"] == 0
+
+
 def test_frustration_cloud_distinct_states():
     """f.2 (Fig. 2, L81/L86): distinct nearest balanced states over many
     trees, counted from the per-tree state signatures, equal the oracle's."""
