@@ -376,24 +376,33 @@ def test_c4_epinions_tree_subset():
 
 @pytest.mark.slow
 def test_c3_amazon_sampled_trees():
-    """C3 (10M / 22M) at full size in bench's batch configuration: per-tree
-    statistics of the whole batch against invariants, and two sampled trees
-    bit-exact against the oracle."""
+    """C3 (10M / 22M) at full size in bench's launch configuration (one step:
+    100 trees as MS-BFS batches of 64 + 36, one tree per labelling launch):
+    per-tree statistics of all trees against invariants, and four sampled
+    trees (first / last of each batch) bit-exact against the oracle -- cycle
+    lengths, depth and the signature of the switched edge set."""
     g, T, _ = graphgen.config("c3")
+    assert T == 100
     graphb.load_graph(g)
-    cnt, agree = graphb.balance_host(8, 1)
+    cnt, agree = graphb.balance_host(T, 1)      # bench's step: batches of 64 + 36 trees
+    st = graphb.stats()
+    assert st["batch"] == 64 and st["batches"] == 2
     ids, per = graphb.tree_stats()
     og = oracle.Graph.from_csr(g)
     c = og.ncomp
     assert np.all(per[:, 1] == g.m - g.n + c)                  # L112
-    assert np.all(agree <= 16) and cnt.max() <= 8
-    for t in (0, 5):
+    assert np.all(agree <= 2 * T) and cnt.max() <= T
+    # sampled trees of both batches (first / last of each): cycle lengths,
+    # depth and the signature of the switched edge set, bit-exact
+    for t in (0, 63, 64, 99):
         parent, dist, _ = og.bfs_tree(1, t)
         flip, sk, nc, md = og.balance_tree(parent)
         assert per[t, 0] == sk and per[t, 2] == md
-        d = graphb.tree_debug(t, 1)
-        assert np.array_equal(d["parent"], parent)
-        assert np.array_equal(d["flip"], flip)
+        assert per[t, 3] == oracle.state_signature(flip)
+    d = graphb.tree_debug(5, 1)
+    parent, _, _ = og.bfs_tree(1, 5)
+    assert np.array_equal(d["parent"], parent)
+    assert np.array_equal(d["flip"], og.balance_tree(parent)[0])
 
 
 @pytest.mark.parametrize("which", ["er", "forest", "c2"])
