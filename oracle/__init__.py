@@ -47,7 +47,6 @@ def lib():
         L.or_splitmix64_next.restype = u64; L.or_splitmix64_next.argtypes = [ctypes.POINTER(u64)]
         L.or_tkey.restype = u64; L.or_tkey.argtypes = [u64, i64]
         L.or_rkey.restype = u64; L.or_rkey.argtypes = [u64, i64, i64]
-        L.or_ekey.restype = u64; L.or_ekey.argtypes = [u64, i64, i64]
         L.or_pscore.restype = ctypes.c_uint32
         L.or_pscore.argtypes = [u64, i64, ctypes.c_int32, ctypes.c_int32]
         L.or_build.restype = ctypes.c_int
@@ -70,6 +69,7 @@ def lib():
         L.or_balance_m.restype = ctypes.c_int
         L.or_balance_m.argtypes = [P, i64, i64, i64, u64, ctypes.c_int, P, P, P]
         L.or_wdraw.restype = u64; L.or_wdraw.argtypes = [u64, i64, ctypes.c_int32, ctypes.c_uint32]
+        L.or_dstart.restype = u64; L.or_dstart.argtypes = [u64, i64, ctypes.c_int32]
         L.or_dfs_tree.restype = ctypes.c_int
         L.or_dfs_tree.argtypes = [P, u64, i64, P]
         L.or_wilson_tree.restype = ctypes.c_int
@@ -99,16 +99,16 @@ def rkey(seed, t, c):
     return int(lib().or_rkey(seed, t, c))
 
 
-def ekey(seed, t, e):
-    return int(lib().or_ekey(seed, t, e))
-
-
 def pscore(seed, t, a, b):
     return int(lib().or_pscore(seed, t, a, b))
 
 
 def wdraw(seed, t, u, j):
     return int(lib().or_wdraw(seed & (2**64 - 1), t, u, j))
+
+
+def dstart(seed, t, u):
+    return int(lib().or_dstart(seed & (2**64 - 1), t, u))
 
 
 def state_signature(flip):

@@ -70,11 +70,6 @@ uint64_t or_rkey(uint64_t seed, int64_t t, int64_t comp)
     return or_mix64(or_tkey(seed, t) ^ (0xD1B54A32D192ED03ULL * (uint64_t)(comp + 1)));
 }
 
-uint64_t or_ekey(uint64_t seed, int64_t t, int64_t eid)
-{
-    return or_mix64(or_tkey(seed, t) + OR_GOLDEN * (uint64_t)(eid + 1));
-}
-
 /* Parent score of the edge {a,b} in tree t (reading R4): the high 32 bits of
  * mix64(tkey + G * (min(a,b) * 2^32 + max(a,b))). */
 uint32_t or_pscore(uint64_t seed, int64_t t, int32_t a, int32_t b)

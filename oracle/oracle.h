@@ -31,7 +31,6 @@ uint64_t or_mix64(uint64_t z);
 uint64_t or_splitmix64_next(uint64_t *state);
 uint64_t or_tkey(uint64_t seed, int64_t t);
 uint64_t or_rkey(uint64_t seed, int64_t t, int64_t comp);
-uint64_t or_ekey(uint64_t seed, int64_t t, int64_t eid);
 uint32_t or_pscore(uint64_t seed, int64_t t, int32_t a, int32_t b);
 
 /* --- graph ------------------------------------------------------------- */

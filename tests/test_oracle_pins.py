@@ -14,6 +14,7 @@ import pytest
 import graphgen
 import oracle
 from tests import _brute as bf
+from tests.test_oracle_spec_pins import spec_rkey
 
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
 
@@ -106,11 +107,11 @@ def test_bfs_dist_and_minhash_parent(seed):
     eid = {(u, v): i for i, (u, v, _) in enumerate(edges)}
     for t in range(4):
         parent, dist, peid = og.bfs_tree(seed, t)
-        # roots: cverts_C[rkey mod |C|]
+        # roots: cverts_C[rkey mod |C|], rkey restated from reading R4
         roots = []
         for c in range(og.ncomp):
             sz = int(coff[c + 1] - coff[c])
-            roots.append(int(cverts[int(coff[c]) + oracle.rkey(seed, t, c) % sz]))
+            roots.append(int(cverts[int(coff[c]) + spec_rkey(seed, t, c) % sz]))
         assert sorted(roots) == sorted(np.flatnonzero(parent == -1).tolist())
         # textbook multi-source BFS
         d = [-1] * g.n
