@@ -19,10 +19,20 @@
  * Conventions:
  *   - m counts undirected edges; the CSR has 2m slots (Table 1, R2).
  *   - eid(u,v) = rank of (min(u,v), max(u,v)) in lexicographic order.
- *   - The tree of index t is defined by (graph, seed, t) only: root of
- *     component C = C's vertices (ascending) [rkey(seed,t,C) mod |C|]; BFS
- *     distances; parent(w) = neighbour one level up whose edge has the
- *     minimum ekey(seed,t,eid) (R4).  Disconnected inputs are forests (R3).
+ *   - The tree of index t is defined by (graph, seed, t) only (reading R4;
+ *     the paper samples "random BFS trees", L479, and gives no rule).  With
+ *     mix64 = the SplitMix64 output function (z ^= z>>30; z *= 0xBF58476D1CE4E5B9;
+ *     z ^= z>>27; z *= 0x94D049BB133111EB; z ^= z>>31, all mod 2^64) and
+ *     G = 0x9E3779B97F4A7C15:
+ *       tkey(seed,t)  = mix64(seed + G*(t+1))
+ *       root of component C (components ranked by their smallest vertex) =
+ *         C's vertices in ascending order [mix64(tkey ^ 0xD1B54A32D192ED03*(C+1)) mod |C|]
+ *       dist = BFS distance from the roots (level-synchronous BFS, L116, L123)
+ *       parent(w) = the neighbour u with dist(u) = dist(w) - 1 minimising the
+ *         pair (pscore(u,w), u), where pscore(u,w) = high 32 bits of
+ *         mix64(tkey + G*(min(u,w)*2^32 + max(u,w))) (original vertex ids;
+ *         ties to the smaller u).
+ *     Disconnected inputs are forests (R3).
  *   - A non-tree edge gets the sign that makes its fundamental cycle even
  *     (L214): flip(e) = (#negative tree edges on the path + neg(e)) mod 2 (R1).
  *
@@ -74,7 +84,12 @@ void gb_free(void);
  * DEVICE outputs on the loaded graph's device, ACCUMULATED (+=):
  *   d_edge_cnt [m] int32, d_vertex_agree [n] int32.
  * cuda_stream: a cudaStream_t to run on (NULL = the library's own stream).
- * Asynchronous with respect to the host when cuda_stream is given. */
+ * Asynchronous with respect to the host: the call enqueues its kernels on
+ * the stream and returns without synchronising (its statistics are read back
+ * by the next gb_get_stats / gb_tree_stats / gb_cloud_states, which wait for
+ * the stream).  Calls share the library's tree workspace: issue successive
+ * calls on one stream, or synchronise between streams.  The first call on a
+ * new graph or batch size allocates (cudaMalloc, which synchronises). */
 int gb_balance_range(int64_t t_begin, int64_t t_end, int64_t t_stride, uint64_t seed,
                      int32_t *d_edge_cnt, int32_t *d_vertex_agree, void *cuda_stream);
 
@@ -94,11 +109,11 @@ int gb_tree_debug(int64_t t, uint64_t seed, int32_t *parent, int32_t *dist,
 int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
                           uint64_t *sum_cycle_len, int64_t *num_cycles);
 
-/* Options (before gb_balance*): "batch" trees per batch (0 = auto),
+/* Options (before gb_balance*): "batch" trees per batch (0 = auto; at most
+ * 64, the multi-source BFS width -- larger values are clamped to 64),
  * "cycle_group" trees per cycle-kernel pass (0 = auto), "walk"
  * (0 = two-ended interval walk, 1 = Alg. 3 descent with warp ballots),
- * "timing" (1 = record per-phase CUDA events), "graphs" (1 = CUDA graphs),
- * "sub" (trees per labelling launch, 0 = auto), "msprof" (see gb_msbfs_profile),
+ * "timing" (1 = record per-phase CUDA events), "sub" (trees per labelling launch, 0 = auto), "msprof" (see gb_msbfs_profile),
  * "recpass" (walk 0: 1 = pre-indexed records scattered in a pass after the
  * top-down pass, 0 = inside it), "jump" (walk 0: 1, 2 or 4 tree levels per
  * ancestor record of the cycle walk), "persist" (bytes of an L2 persisting
@@ -115,7 +130,8 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
  * popping), "reset" (every option back to its default). */
 int gb_set_option(const char *key, int64_t value);
 
-/* Statistics of the last gb_balance / gb_balance_range call:
+/* Statistics of the last gb_balance / gb_balance_range call (waits for its
+ * stream); the totals cover every tree of the call:
  * ints[0] trees, [1] sum of cycle lengths, [2] cycles, [3] kernel launches,
  * [4] batches, [5] max tree depth, [6] batch size used, [7] cycle group used,
  * [8] edges of some Sigma_T that contradict the L224 bipartition (option
@@ -139,6 +155,14 @@ int gb_get_stats(int64_t *ints, int n_ints, double *phase_ms, int n_phase);
  * 2^-64 collisions -- frustration-cloud analytics, Fig. 2 L81/L86);
  * tree_ids[i] = t.  Returns the count. */
 int64_t gb_tree_stats(uint64_t *out, int64_t *tree_ids, int64_t max_trees);
+
+/* Frustration-cloud analytics (f.2, Fig. 2 L81/L86: "5 unique states"): the
+ * distinct nearest balanced states among the trees gb_tree_stats records,
+ * counted on the device (hash table over the state signatures).  Writes
+ * min(k, max_states) pairs sig[i] / count[i] (trees reaching that state;
+ * any order) and returns k, the number of distinct states (negative
+ * gb_err on failure).  sig or count may be NULL. */
+int64_t gb_cloud_states(uint64_t *sig, uint64_t *count, int64_t max_states);
 
 /* Profiling aid: with option "msprof" = 1, the multi-source BFS of the last
  * batch records %globaltimer (ns) at its phase boundaries, out[4*L + k] for

@@ -67,6 +67,15 @@ struct Stats {
     double phase_ms[GB_NPHASE] = {0};
     std::vector<uint64_t> per_tree;   // 4 per recorded tree
     std::vector<int64_t> tree_ids;
+    // gb_balance_range returns without synchronising: the device-side totals,
+    // per-tree records and phase events of the call are read back lazily, by
+    // the first gb_get_stats / gb_tree_stats / gb_cloud_states afterwards
+    bool pending = false;
+    cudaStream_t stream = nullptr;
+    int64_t nrec = 0;
+    bool harary = false;
+    std::vector<cudaEvent_t> evs;      // (GB_NPHASE + 1) per batch when "timing" is set
+    double sample_ms = 0;
 };
 
 struct State {
@@ -79,6 +88,8 @@ struct State {
     int32_t *d_given = nullptr;                    // caller tree (gb_balance_given_tree)
     unsigned long long *d_visited = nullptr;       // [kMaxBatch]
     unsigned long long *d_rec_stats = nullptr;     // [kRecCap][4]
+    unsigned long long *d_tot = nullptr;           // [4] sum k, cycles, max depth over every tree of the call
+    unsigned long long *d_states = nullptr;        // gb_cloud_states: hash table [2 * kStateSlots]
     unsigned long long *d_hbad = nullptr;          // option "harary": violations found
     std::vector<int32_t> h_comp;
     size_t free_at_load = 0;   // device memory free after ingest (cudaMemGetInfo costs ~2 ms)
@@ -87,6 +98,7 @@ struct State {
 };
 static State S;
 constexpr int64_t kRecCap = 1 << 16;  // per-tree statistics kept for gb_tree_stats
+constexpr int64_t kStateSlots = 2 * kRecCap;  // open-addressing table of gb_cloud_states
 
 static void free_ws(Workspace &w) {
     void *ptrs[] = {w.vst, w.qv, w.qs, w.qr, w.pkeyq, w.lvl, w.vbase, w.size, w.sz64,
@@ -196,8 +208,14 @@ __global__ void k_tree_keys(uint64_t *tkey, int B, uint64_t seed, int64_t t0, in
 }
 
 __global__ void k_record_stats(const unsigned long long *tstat, const int32_t *depth, int B,
-                               unsigned long long *rec, int64_t pos, int64_t cap) {
+                               unsigned long long *rec, int64_t pos, int64_t cap,
+                               unsigned long long *tot) {
     int b = threadIdx.x;
+    if (b < B) {
+        atomicAdd(tot, tstat[3 * b]);
+        atomicAdd(tot + 1, tstat[3 * b + 1]);
+        atomicMax(tot + 2, (unsigned long long)depth[b]);
+    }
     if (b < B && pos + b < cap) {
         rec[4 * (pos + b)] = tstat[3 * b];
         rec[4 * (pos + b) + 1] = tstat[3 * b + 1];
@@ -206,9 +224,29 @@ __global__ void k_record_stats(const unsigned long long *tstat, const int32_t *d
     }
 }
 
+// f.2: distinct nearest balanced states among the recorded trees.  Open
+// addressing over the 64-bit state signatures (rec[4i+3]); slot = {sig, count}
+// with sig 0 = empty (the signature of "no switched edge" is 0 as well, so it
+// is kept in a dedicated counter, zero[0]).
+__global__ void k_cloud_states(const unsigned long long *rec, int64_t k, unsigned long long *tab,
+                               int64_t slots, unsigned long long *zero) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < k;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const unsigned long long sig = rec[4 * i + 3];
+        if (sig == 0) { atomicAdd(zero, 1ull); continue; }
+        int64_t h = (int64_t)(mix64(sig) & (uint64_t)(slots - 1));
+        for (;;) {
+            const unsigned long long prev = atomicCAS(tab + 2 * h, 0ull, sig);
+            if (prev == 0 || prev == sig) { atomicAdd(tab + 2 * h + 1, 1ull); break; }
+            h = (h + 1) & (slots - 1);
+        }
+    }
+}
+
 static int auto_batch(int64_t ntrees) {
     if (S.opt.sampler != 0) return 1;   // sampled trees go one at a time (caller-tree path)
-    if (S.opt.batch > 0) return (int)std::min<int64_t>(S.opt.batch, kMaxBatch);
+    // the multi-source BFS holds one bit per tree in a 64-bit word
+    if (S.opt.batch > 0) return (int)std::min<int64_t>(S.opt.batch, kMsBatch);
     const size_t have = S.free_at_load;
     int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk == 1));
     int64_t b = std::min<int64_t>({ntrees, (int64_t)kMsBatch, std::max<int64_t>(bm, 1)});
@@ -234,10 +272,56 @@ static int auto_group(int B) {
 }
 
 // the whole hot path over trees t_begin, t_begin+stride, ... < t_end
+static void drop_events(Stats &T) {
+    for (auto e : T.evs) cudaEventDestroy(e);   // released once complete
+    T.evs.clear();
+}
+
+// read back what the last balance_range left on the device (synchronises
+// with its stream once)
+static int finalize_stats() {
+    Stats &T = S.st;
+    if (!T.pending) return GB_OK;
+    T.pending = false;
+    GB_CUDA_TRY(cudaStreamSynchronize(T.stream));
+    unsigned long long tot[4] = {0, 0, 0, 0};
+    GB_CUDA_TRY(cudaMemcpy(tot, S.d_tot, sizeof(tot), cudaMemcpyDeviceToHost));
+    T.sumk = tot[0];
+    T.cycles = tot[1];
+    T.max_depth = (int64_t)tot[2];
+    T.per_tree.resize(4 * T.nrec);
+    if (T.nrec)
+        GB_CUDA_TRY(cudaMemcpy(T.per_tree.data(), S.d_rec_stats, sizeof(uint64_t) * 4 * T.nrec,
+                               cudaMemcpyDeviceToHost));
+    if (T.harary) {
+        unsigned long long hb = 0;
+        GB_CUDA_TRY(cudaMemcpy(&hb, S.d_hbad, sizeof(hb), cudaMemcpyDeviceToHost));
+        T.harary_bad = (int64_t)hb;
+    }
+    for (size_t base = 0; base + GB_NPHASE < T.evs.size(); base += GB_NPHASE + 1) {
+        for (int i = 0; i < GB_NPHASE; i++) {
+            float ms = 0;
+            cudaEventElapsedTime(&ms, T.evs[base + i], T.evs[base + i + 1]);
+            T.phase_ms[i] += ms;
+        }
+    }
+    drop_events(T);
+    T.phase_ms[GB_PHASE_BFS] += T.sample_ms;
+    return GB_OK;
+}
+
 static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_t seed,
                          int32_t *d_cnt, int32_t *d_agree, cudaStream_t st) {
     Stats &T = S.st;
+    drop_events(T);   // an unread previous call is discarded
     T = Stats();
+    T.stream = st;
+    if (!S.d_rec_stats) {
+        GB_CUDA_TRY(cudaMalloc(&S.d_rec_stats, sizeof(unsigned long long) * 4 * kRecCap));
+        GB_CUDA_TRY(cudaMalloc(&S.d_tot, sizeof(unsigned long long) * 4));
+    }
+    GB_CUDA_TRY(cudaMemsetAsync(S.d_tot, 0, sizeof(unsigned long long) * 4, st));
+    T.pending = true;
     const int64_t K = t_end > t_begin ? (t_end - t_begin + stride - 1) / stride : 0;
     if (K == 0) return GB_OK;
     const bool descent = S.opt.walk == 1;
@@ -265,17 +349,14 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     if (S.ws.msprof) GB_CUDA_TRY(cudaMemsetAsync(S.ws.msprof, 0, sizeof(unsigned long long) * 2048, st));
     T.batch_used = B;
     T.group_used = G;
-    if (!S.d_rec_stats) {
-        GB_CUDA_TRY(cudaMalloc(&S.d_rec_stats, sizeof(unsigned long long) * 4 * kRecCap));
-    }
-    std::vector<cudaEvent_t> evs;
+    std::vector<cudaEvent_t> &evs = T.evs;
     const bool timing = S.opt.timing != 0;
     int64_t done = 0;
     // uniform sampler: trees per sampling chunk (<= kMaxBatch, ~2 GB of walk state)
     const int64_t Wc = std::max<int64_t>(1, std::min<int64_t>({(int64_t)kMaxBatch, K,
                                              (int64_t)(2.0e9 / (13.0 * (double)S.g.n))}));
     cudaEvent_t wev[2];
-    double sample_ms = 0;
+    double &sample_ms = T.sample_ms;
     while (done < K) {
         const int nb = (int)std::min<int64_t>(B, K - done);
         const int64_t t0 = t_begin + done * stride;
@@ -336,47 +417,24 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[6], st));
         if (done < kRecCap) {
-            k_record_stats<<<1, kMaxBatch, 0, st>>>(S.ws.tstat, S.ws.depth, nb, S.d_rec_stats, done, kRecCap);
-            ++T.launches;
             for (int b = 0; b < nb && done + b < kRecCap; b++) T.tree_ids.push_back(t0 + b * stride);
         }
+        k_record_stats<<<1, kMaxBatch, 0, st>>>(S.ws.tstat, S.ws.depth, nb, S.d_rec_stats, done, kRecCap,
+                                                S.d_tot);
+        ++T.launches;
         done += nb;
         T.batches++;
     }
     GB_CUDA_TRY(cudaGetLastError());
-    if (S.opt.harary) {
-        unsigned long long hb = 0;
-        GB_CUDA_TRY(cudaMemcpyAsync(&hb, S.d_hbad, sizeof(hb), cudaMemcpyDeviceToHost, st));
-        GB_CUDA_TRY(cudaStreamSynchronize(st));
-        T.harary_bad = (int64_t)hb;
-    }
-    const int64_t nrec = std::min<int64_t>(K, kRecCap);
-    T.per_tree.resize(4 * nrec);
-    GB_CUDA_TRY(cudaMemcpyAsync(T.per_tree.data(), S.d_rec_stats, sizeof(uint64_t) * 4 * nrec,
-                                cudaMemcpyDeviceToHost, st));
-    GB_CUDA_TRY(cudaStreamSynchronize(st));
+    T.harary = S.opt.harary != 0;
+    T.nrec = std::min<int64_t>(K, kRecCap);
     T.trees = K;
-    for (int64_t i = 0; i < nrec; i++) {
-        T.sumk += T.per_tree[4 * i];
-        T.cycles += T.per_tree[4 * i + 1];
-        T.max_depth = std::max<int64_t>(T.max_depth, (int64_t)T.per_tree[4 * i + 2]);
-    }
-    if (timing) {
-        for (size_t base = 0; base < evs.size(); base += GB_NPHASE + 1) {
-            for (int i = 0; i < GB_NPHASE; i++) {
-                float ms = 0;
-                cudaEventElapsedTime(&ms, evs[base + i], evs[base + i + 1]);
-                T.phase_ms[i] += ms;
-            }
-        }
-        for (auto e : evs) cudaEventDestroy(e);
-        T.phase_ms[GB_PHASE_BFS] += sample_ms;
-    }
-    return GB_OK;
+    return GB_OK;   // no host synchronisation (statistics are read lazily)
 }
 
 static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
     Stats &T = S.st;
+    drop_events(T);
     T = Stats();
     int rc = ensure_workspace(1, S.opt.walk == 1);
     if (rc) return rc;
@@ -469,10 +527,13 @@ static void release_graph(bool keep_ws) {
 }
 
 void gb_free(void) {
+    drop_events(S.st);
     release_graph(false);
     arena_free_all();
     if (S.d_visited) cudaFree(S.d_visited);
     if (S.d_rec_stats) cudaFree(S.d_rec_stats);
+    if (S.d_tot) cudaFree(S.d_tot);
+    if (S.d_states) cudaFree(S.d_states);
     if (S.d_hbad) cudaFree(S.d_hbad);
     if (S.stream) cudaStreamDestroy(S.stream);
     Options keep = S.opt;
@@ -579,7 +640,6 @@ int gb_set_option(const char *key, int64_t value) {
         }
         S.opt.persist = value;
     }
-    else if (!strcmp(key, "graphs")) { /* reserved */ }
     else { set_error(std::string("unknown option ") + key); return GB_EINVAL; }
     return GB_OK;
 }
@@ -673,6 +733,7 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip, uint64_t *sum_cy
 }
 
 int gb_get_stats(int64_t *ints, int n_ints, double *phase_ms, int n_phase) {
+    if (finalize_stats()) return GB_ECUDA;
     const Stats &T = S.st;
     int64_t v[9] = {T.trees, (int64_t)T.sumk, (int64_t)T.cycles, T.launches, T.batches,
                     T.max_depth, T.batch_used, T.group_used, T.harary_bad};
@@ -695,7 +756,39 @@ int gb_label_profile(uint64_t *out) {
     return GB_OK;
 }
 
+int64_t gb_cloud_states(uint64_t *sig, uint64_t *count, int64_t max_states) {
+    if (finalize_stats()) return GB_ECUDA;
+    const Stats &T = S.st;
+    if (!S.d_rec_stats || T.nrec == 0) return 0;
+    if (!S.d_states) {
+        cudaError_t e = cudaMalloc(&S.d_states, sizeof(unsigned long long) * (2 * kStateSlots + 1));
+        if (e != cudaSuccess) { set_error(std::string("cudaMalloc states: ") + cudaGetErrorString(e)); S.d_states = nullptr; return GB_ENOMEM; }
+    }
+    cudaStream_t st = S.stream;
+    if (cudaMemsetAsync(S.d_states, 0, sizeof(unsigned long long) * (2 * kStateSlots + 1), st) != cudaSuccess) return GB_ECUDA;
+    k_cloud_states<<<(unsigned)((T.nrec + 255) / 256), 256, 0, st>>>(S.d_rec_stats, T.nrec, S.d_states, kStateSlots,
+                                                                     S.d_states + 2 * kStateSlots);
+    std::vector<unsigned long long> tab(2 * kStateSlots + 1);
+    if (cudaMemcpyAsync(tab.data(), S.d_states, sizeof(unsigned long long) * tab.size(), cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+        cudaStreamSynchronize(st) != cudaSuccess) {
+        set_error("gb_cloud_states: copy failed");
+        return GB_ECUDA;
+    }
+    int64_t k = 0;
+    if (tab[2 * kStateSlots]) {
+        if (k < max_states) { if (sig) sig[k] = 0; if (count) count[k] = tab[2 * kStateSlots]; }
+        k++;
+    }
+    for (int64_t h = 0; h < kStateSlots; h++) {
+        if (!tab[2 * h]) continue;
+        if (k < max_states) { if (sig) sig[k] = tab[2 * h]; if (count) count[k] = tab[2 * h + 1]; }
+        k++;
+    }
+    return k;
+}
+
 int64_t gb_tree_stats(uint64_t *out, int64_t *tree_ids, int64_t max_trees) {
+    if (finalize_stats()) return GB_ECUDA;
     const Stats &T = S.st;
     int64_t k = std::min<int64_t>(max_trees, (int64_t)T.tree_ids.size());
     for (int64_t i = 0; i < k; i++) {

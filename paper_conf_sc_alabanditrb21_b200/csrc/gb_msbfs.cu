@@ -738,8 +738,10 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
 int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStream_t st,
               int64_t *launches) {
     if (B < 1 || B > kMsBatch) { set_error("msbfs: batch out of range"); return GB_EINVAL; }
-    static int blocks = 0;
-    if (!blocks) {
+    // co-resident grid size, recomputed when the device changes (SM count)
+    static int blocks = 0, blocks_dev = -1;
+    if (blocks_dev != g.dev) {
+        blocks_dev = g.dev;
         int per = 0;
         GB_CUDA_TRY(cudaFuncSetAttribute(k_msbfs, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMsSmem));
         if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_msbfs, kBlock, kMsSmem) != cudaSuccess || per < 1)

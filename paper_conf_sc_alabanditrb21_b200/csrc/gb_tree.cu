@@ -881,8 +881,10 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
                    cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub,
                    int recpass, size_t persist, int sampler) {
     if (descent) recpass = 0;
-    static int bfs_blocks = 0, up_blocks[2] = {0, 0}, down_blocks[2] = {0, 0};
-    if (!bfs_blocks) {
+    // co-resident grid sizes, recomputed when the device changes
+    static int bfs_blocks = 0, up_blocks[2] = {0, 0}, down_blocks[2] = {0, 0}, blocks_dev = -1;
+    if (blocks_dev != g.dev) {
+        blocks_dev = g.dev;
         bfs_blocks = coop_blocks((const void *)k_bfs, g.num_sms);
         up_blocks[0] = coop_blocks((const void *)k_bottom_up<false>, g.num_sms);
         up_blocks[1] = coop_blocks((const void *)k_bottom_up<true>, g.num_sms);

@@ -57,6 +57,7 @@ def lib():
         "gb_set_option": (i32, [ctypes.c_char_p, i64]),
         "gb_get_stats": (i32, [P, i32, P, i32]),
         "gb_tree_stats": (i64, [P, P, i64]),
+        "gb_cloud_states": (i64, [P, P, i64]),
         "gb_msbfs_profile": (i32, [P]),
         "gb_label_profile": (i32, [P]),
         "gb_graph_info": (i32, [P, P, P]),
@@ -76,7 +77,7 @@ def exported_symbols():
     return ["gb_load_csr", "gb_balance", "gb_free", "gb_balance_range", "gb_tree_debug",
             "gb_balance_given_tree", "gb_set_option", "gb_get_stats", "gb_tree_stats",
             "gb_graph_info", "gb_graph_debug", "gb_selftest", "gb_last_error", "gb_msbfs_profile",
-            "gb_label_profile"]
+            "gb_label_profile", "gb_cloud_states"]
 
 
 def _check(rc):
@@ -166,41 +167,52 @@ def balance_range(t_begin, t_end, t_stride, seed, d_edge_cnt, d_vertex_agree, st
 
 
 def balance(num_trees, seed, group=None):
-    """The frustration cloud over trees 0..num_trees-1 (Alg. 2).
+    """The frustration cloud over trees 0..num_trees-1 (Alg. 2): host numpy
+    arrays (edge_flip_counts uint32[m], vertex_agree uint32[n]).
 
-    Without an initialised torch.distributed group this is gb_balance (host
-    outputs).  With one, rank r balances trees {t : t mod W == r} into int32
-    device counters and one all-reduce(SUM) merges them; every rank returns
-    the same arrays.
+    Without an initialised torch.distributed group this is gb_balance.  With
+    one, rank r balances trees {t : t mod W == r} into one int32 device buffer
+    [cnt | agree] and one all-reduce(SUM) merges the shards (PAPER.md L248);
+    every rank returns the same arrays, of the same type as without a group.
     """
     import torch.distributed as dist
     if not (dist.is_available() and dist.is_initialized()):
         return balance_host(num_trees, seed)
-    return sharded_balance(num_trees, seed, dist.get_rank(group), dist.get_world_size(group),
-                           _device_range, group=group)
+    _, m, _ = graph_info()
+    cnt, agree = sharded_balance(num_trees, seed, dist.get_rank(group), dist.get_world_size(group),
+                                 _device_range, m, group=group)
+    return (cnt.cpu().numpy().astype(np.uint32), agree.cpu().numpy().astype(np.uint32))
+
+
+def counter_buffer(device=None):
+    """One int32 device buffer [edge counters (m) | vertex agree (n)]: the
+    layout of the all-reduce, so no concatenation is needed per call."""
+    import torch
+    n, m, _ = graph_info()
+    dev = device if device is not None else torch.device("cuda", torch.cuda.current_device())
+    return torch.zeros(m + n, dtype=torch.int32, device=dev)
+
+
+def balance_range_buf(t_begin, t_end, t_stride, seed, buf, stream=None):
+    """gb_balance_range into a counter_buffer() (accumulating)."""
+    _, m, _ = graph_info()
+    balance_range(t_begin, t_end, t_stride, seed, buf[:m], buf[m:], stream)
 
 
 def _device_range(t_begin, t_end, stride, seed):
-    import torch
-    n, m, _ = graph_info()
-    dev = torch.device("cuda", torch.cuda.current_device())
-    cnt = torch.zeros(max(m, 1), dtype=torch.int32, device=dev)
-    agree = torch.zeros(n, dtype=torch.int32, device=dev)
-    balance_range(t_begin, t_end, stride, seed, cnt, agree)
-    return cnt, agree
+    buf = counter_buffer()
+    balance_range_buf(t_begin, t_end, stride, seed, buf)
+    return buf
 
 
-def sharded_balance(num_trees, seed, rank, world, range_fn, group=None):
+def sharded_balance(num_trees, seed, rank, world, range_fn, m, group=None):
     """Host logic of the multi-GPU path, independent of the
     backend: rank computes its tree shard with range_fn(t_begin, t_end,
-    stride, seed) -> (cnt, agree) tensors, then one all_reduce(SUM) of the
-    concatenated [cnt | agree] buffer."""
-    import torch
+    stride, seed) -> one int32 tensor [cnt (m) | agree (n)], then one
+    all_reduce(SUM) of that buffer in place.  Returns (cnt, agree) views."""
     import torch.distributed as dist
-    cnt, agree = range_fn(rank, num_trees, world, seed)
-    buf = torch.cat([cnt.reshape(-1), agree.reshape(-1)])
+    buf = range_fn(rank, num_trees, world, seed)
     dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=group)
-    m = cnt.numel()
     return buf[:m], buf[m:]
 
 
@@ -251,13 +263,18 @@ def tree_stats(max_trees=1 << 16):
     return ids[:k], out[: 4 * k].reshape(k, 4)
 
 
-def cloud_states(max_trees=1 << 16):
-    """Frustration-cloud analytics of the last balance call:
-    {state signature: number of sampled trees reaching that nearest balanced
-    state}.  len() of it is the number of distinct states found."""
-    _, per = tree_stats(max_trees)
-    sigs, counts = np.unique(per[:, 3], return_counts=True)
-    return {int(s): int(c) for s, c in zip(sigs, counts)}
+def cloud_states(max_states=1 << 16):
+    """Frustration-cloud analytics of the last balance call (SURVEY §8 f.2,
+    gb_cloud_states, counted on the device): {state signature: number of
+    sampled trees reaching that nearest balanced state}.  len() of it is the
+    number of distinct states found."""
+    sig = np.zeros(max_states, np.uint64)
+    cnt = np.zeros(max_states, np.uint64)
+    k = lib().gb_cloud_states(_ptr(sig), _ptr(cnt), max_states)
+    if k < 0:
+        _check(int(k))
+    k = min(int(k), max_states)
+    return {int(s): int(c) for s, c in zip(sig[:k], cnt[:k])}
 
 
 def msbfs_profile():

@@ -38,9 +38,9 @@ def _worker(rank, world, port, T, seed, out):
         def range_fn(t_begin, t_end, stride, s):
             seen.append((t_begin, t_end, stride))
             c, a = og.balance(t_end, s, t_begin=t_begin, stride=stride)
-            return torch.from_numpy(c.astype(np.int32)), torch.from_numpy(a.astype(np.int32))
+            return torch.from_numpy(np.concatenate([c, a]).astype(np.int32))
 
-        cnt, agree = sharded_balance(T, seed, rank, world, range_fn)
+        cnt, agree = sharded_balance(T, seed, rank, world, range_fn, g.m)
         assert seen == [(rank, T, world)]
         out[rank] = (cnt.numpy().copy(), agree.numpy().copy())
     finally:
