@@ -163,16 +163,61 @@ def load_peaks():
 
 
 # ---------------------------------------------------------------------------
+def _cpu_model():
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+_ORACLE_SHARED = {}
+
+
+def _oracle_shard(job):
+    """Child of the all-cores baseline (fork): trees t_begin, t_begin+P, ...
+    of the shared oracle graph."""
+    og = _ORACLE_SHARED["og"]
+    t0 = time.perf_counter()
+    og.balance(job[1], job[2], t_begin=job[0], stride=job[3])
+    return time.perf_counter() - t0
+
+
 def cpu_baseline(g, seed, trees, c_nt):
-    """The oracle as it stands (single-threaded C), on a bounded sample."""
+    """The oracle as it stands (plain single-threaded C), on a bounded sample:
+    1 core (`trees` trees), and all host cores as P = nproc independent
+    processes over disjoint tree subsets (P trees, one per process; the
+    graph is built once and shared copy-on-write by fork)."""
+    import multiprocessing as mp
     import oracle
     og = oracle.Graph.from_csr(g)
     t0 = time.perf_counter()
     og.balance(trees, seed)
     dt = time.perf_counter() - t0
-    return {"value": trees * c_nt / dt, "unit": "cycles/s", "cores": 1, "kind": "oracle",
-            "sample": f"{trees} tree(s) of the same workload (seed {seed}), {dt:.2f} s, "
-                      f"single-threaded plain C (-O2)"}
+    out = {"value": trees * c_nt / dt, "unit": "cycles/s", "cores": 1, "kind": "oracle",
+           "cpu_model": _cpu_model(), "host_cores": os.cpu_count(),
+           "sample": f"{trees} tree(s) of the same workload (seed {seed}), {dt:.2f} s, "
+                     f"single-threaded plain C (-O2)"}
+    P = os.cpu_count() or 1
+    if P > 1:
+        try:
+            _ORACLE_SHARED["og"] = og
+            ctx = mp.get_context("fork")
+            with ctx.Pool(P) as pool:
+                t1 = time.perf_counter()
+                pool.map(_oracle_shard, [(r, P, seed, P) for r in range(P)], chunksize=1)
+                dt_all = time.perf_counter() - t1
+            out["all_cores"] = {"value": P * c_nt / dt_all, "unit": "cycles/s", "cores": P,
+                                "sample": f"{P} trees, one per process (tree-parallel oracle, "
+                                          f"fork after the graph build), {dt_all:.2f} s wall"}
+        except Exception as e:  # the 1-core figure stands on its own
+            out["all_cores"] = {"value": None, "error": str(e)[:200]}
+        finally:
+            _ORACLE_SHARED.clear()
+    return out
 
 
 def sample_trees_for(g, requested):
@@ -213,17 +258,38 @@ def run_reference(args, g, desc, T):
     print(json.dumps(line), flush=True)
 
 
+def _relaunch_under_torchrun(args):
+    """`bench.py --gpus N` started without torchrun: start the N ranks here
+    (one process per GPU, 127.0.0.1 rendezvous) and return their exit code."""
+    import socket
+    sock = socket.socket()
+    sock.bind(("127.0.0.1", 0))
+    port = sock.getsockname()[1]
+    sock.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
 def main():
     args = parse()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl == "ours":
+        sys.exit(_relaunch_under_torchrun(args))
     import graphgen
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "ours" and world != args.gpus:
+        raise SystemExit(f"bench.py --gpus {args.gpus} but WORLD_SIZE={world}")
     g, T_default, desc = graphgen.config(args.config)
     T = args.trees or T_default
     if args.impl == "reference":
         return run_reference(args, g, desc, T)
 
+    if world > 1:
+        # rank counts and the NCCL transport in the log (init lines only)
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
     import torch
     import torch.distributed as dist
     from paper_conf_sc_alabanditrb21_b200 import graphb
@@ -241,14 +307,12 @@ def main():
     c_nt = m - n + ncomp
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream(dev)
-    cnt = torch.zeros(max(m, 1), dtype=torch.int32, device=dev)
-    agree = torch.zeros(n, dtype=torch.int32, device=dev)
+    buf = graphb.counter_buffer(dev)      # [cnt (m) | agree (n)]: the all-reduce buffer, allocated once
     total_trees = T * world
 
     def step(seed):
-        graphb.balance_range(rank, total_trees, world, seed, cnt, agree, stream=stream)
+        graphb.balance_range_buf(rank, total_trees, world, seed, buf, stream=stream)
         if world > 1:
-            buf = torch.cat([cnt, agree])
             dist.all_reduce(buf)
 
     for i in range(args.warmup):
@@ -258,52 +322,57 @@ def main():
     step(99)
     phase = graphb.stats()
     graphb.set_option("timing", 0)
+    step(98)
+    launches_per_step = graphb.stats()["launches"]
 
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     clk = ClockSampler(local)
     clk.start()
-    ev0 = torch.cuda.Event(enable_timing=True)
-    ev1 = torch.cuda.Event(enable_timing=True)
-    launches = 0
-    sumk = 0
-    ev0.record(stream)
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
+    evs[0].record(stream)
     for s in range(args.steps):
-        step(1 + s)
-        st = graphb.stats()
-        launches += st["launches"]
-        sumk += st["sum_cycle_len"]
-    ev1.record(stream)
+        step(1 + s)                       # no host synchronisation inside the timed region
+        evs[s + 1].record(stream)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     clocks = clk.stop()
-    ms = ev0.elapsed_time(ev1)
-    t = torch.tensor([ms], dtype=torch.float64, device=dev)
+    ms = evs[0].elapsed_time(evs[-1])
+    step_ms = [evs[s].elapsed_time(evs[s + 1]) for s in range(args.steps)]
+    t = torch.tensor([ms] + step_ms, dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms_max = float(t.item())
+    ms_max = float(t[0].item())
+    step_max = [float(x) for x in t[1:].tolist()]
     cycles_total = args.steps * total_trees * c_nt
     value = cycles_total / (ms_max / 1000.0)
+    per_step_cycles = total_trees * c_nt
+    steps_summary = {"best_ms": min(step_max), "median_ms": statistics.median(step_max),
+                     "best_value": per_step_cycles / (min(step_max) / 1000.0),
+                     "median_value": per_step_cycles / (statistics.median(step_max) / 1000.0),
+                     "note": "per-step CUDA events, max over ranks; best-of and median as the paper's L327"}
 
     # roofline of the dominant phase (from the timed-phase step)
     ph = phase["phase_ms"]
     dom = max(ph, key=lambda k: ph[k])
-    per_tree_sumk = phase["sum_cycle_len"] / max(1, phase["trees"])
-    bytes_per_tree = phase_bytes(n, m, per_tree_sumk * phase["trees"], phase["trees"], phase["batch"])
     trees_in_step = phase["trees"]
-    sub_trees = 1 if (args.sub == 1 or (args.sub == 0 and n >= (1 << 22))) else phase["batch"]
-    launches_of = {"cycles": max(1, phase["batches"] * -(-phase["batch"] // max(1, phase["cycle_group"]))),
-                   "bottom_up": max(1, -(-trees_in_step // sub_trees)),
-                   "top_down": max(1, -(-trees_in_step // sub_trees))}
+    per_tree_sumk = phase["sum_cycle_len"] / max(1, trees_in_step)
+    bytes_per_tree = phase_bytes(n, m, per_tree_sumk * trees_in_step, trees_in_step, phase["batch"])
+    # launches per phase, from the library's own counts (gb_get_stats [6], [7], [9], [10])
+    launches_of = {"bfs": max(1, phase["batches"] * -(-phase["batch"] // max(1, phase["bfs_group"]))),
+                   "cycles": max(1, phase["batches"] * -(-phase["batch"] // max(1, phase["cycle_group"]))),
+                   "bottom_up": max(1, phase["batches"] * -(-phase["batch"] // max(1, phase["sub"]))),
+                   "top_down": max(1, phase["batches"] * -(-phase["batch"] // max(1, phase["sub"])))}
     dom_launches = launches_of.get(dom, phase["batches"])
     dom_bytes_per_launch = bytes_per_tree[dom] * trees_in_step / dom_launches
     dom_ms_per_launch = ph[dom] / dom_launches
     peak, peak_src = load_peaks()
     achieved = dom_bytes_per_launch / (dom_ms_per_launch / 1000.0) / 1e9
-    kernel_of = {"bfs": "k_msbfs", "bottom_up": "k_bottom_up", "top_down": "k_top_down",
-                 "cycles": "k_cycles_two_ended", "accumulate": "k_accumulate_edges", "init": "k_ms_roots"}
+    bfs_kernel = "k_tbfs" if any(kv.replace(" ", "") == "bfs=0" for kv in args.opt) else "k_msbfs"
+    kernel_of = {"bfs": bfs_kernel, "bottom_up": "k_bottom_up", "top_down": "k_top_down",
+                 "cycles": "k_cycles_two_ended", "accumulate": "k_accumulate_edges", "init": "k_tb_roots"}
     traffic = ncu_traffic(args.config, kernel_of[dom], trees_in_step / dom_launches)
     path_bytes = sum(bytes_per_tree.values()) * total_trees * args.steps / world
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -312,15 +381,19 @@ def main():
                 "path_achieved": path_bytes / (ms_max / 1000.0) / 1e9,
                 "path_frac": path_bytes / (ms_max / 1000.0) / 1e9 / peak,
                 "bytes_per_launch": dom_bytes_per_launch, "launch_ms": dom_ms_per_launch,
+                "traffic_source": "profiles/traffic_%s.json (ncu --set full, per launch)" % args.config,
                 "phase_share": {k: v / max(1e-9, sum(ph.values())) for k, v in ph.items()}}
+    graphb_only = (ph["bottom_up"] + ph["top_down"] + ph["cycles"]) / max(1, trees_in_step)
 
-    # end-to-end through the public API with host buffers (rank-local)
+    # end-to-end through the public API with host buffers: gb_load_csr (H2D +
+    # ingest) + gb_balance (host outputs; N > 1: graphb.balance, the sharded
+    # path with its all-reduce) per step
     e2e = None
     if not args.no_e2e:
         pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory().numpy()
         hrp, hcol, hsg = pin(g.row_ptr), pin(g.col), pin(g.sign)
-        h_cnt = torch.empty(max(m, 1), dtype=torch.int32).pin_memory()
-        h_agr = torch.empty(n, dtype=torch.int32).pin_memory()
+        h_cnt = torch.empty(max(m, 1), dtype=torch.int32).pin_memory().numpy().view(np.uint32)
+        h_agr = torch.empty(n, dtype=torch.int32).pin_memory().numpy().view(np.uint32)
         e_steps = max(1, min(args.steps, 3))
         if world > 1:
             dist.barrier()
@@ -331,16 +404,13 @@ def main():
             ta = time.perf_counter()
             graphb.load_csr(hrp, hcol, hsg)
             tb = time.perf_counter()
-            cnt.zero_(); agree.zero_()
-            step(500 + s)
+            if world > 1:
+                graphb.balance(total_trees, 500 + s)
+            else:
+                graphb.balance_host(T, 500 + s, out=(h_cnt, h_agr))
             if trace:
-                torch.cuda.synchronize()
-            tc = time.perf_counter()
-            h_cnt.copy_(cnt); h_agr.copy_(agree)
-            torch.cuda.synchronize()
-            if trace:
-                print(f"e2e step {s}: load {1e3 * (tb - ta):.1f} ms, balance {1e3 * (tc - tb):.1f} ms, "
-                      f"d2h {1e3 * (time.perf_counter() - tc):.1f} ms", file=sys.stderr, flush=True)
+                print(f"e2e step {s}: load {1e3 * (tb - ta):.1f} ms, balance+d2h "
+                      f"{1e3 * (time.perf_counter() - tb):.1f} ms", file=sys.stderr, flush=True)
         el = time.perf_counter() - t0
         tt = torch.tensor([el], dtype=torch.float64, device=dev)
         if world > 1:
@@ -348,10 +418,11 @@ def main():
         e2e = {"value": e_steps * total_trees * c_nt / float(tt.item()), "unit": "cycles/s",
                "h2d_bytes_per_step": int(hrp.nbytes + hcol.nbytes + hsg.nbytes),
                "d2h_bytes_per_step": int(4 * (m + n)),
-               "note": "per step: gb_load_csr (H2D + ingest) + balance + D2H of the counters"}
+               "note": "per step: gb_load_csr (H2D + ingest) + gb_balance with host outputs "
+                       "(N > 1: graphb.balance = shard + NCCL all-reduce + D2H)"}
 
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if rank == 0 and not args.no_cpu_baseline:
         if g.m > 2e8 and not args.cpu_sample_trees:
             # the single-threaded oracle needs minutes just to build a 1 B-edge graph
             cpu = {"value": None, "unit": "cycles/s", "cores": 1, "kind": "oracle",
@@ -371,6 +442,7 @@ def main():
             "config": {"workload": f"{args.config}: {desc}", "n": n, "m": m, "components": ncomp,
                        "cycles_per_tree": c_nt, "trees_per_gpu": T, "trees_total": total_trees,
                        "batch": phase["batch"], "cycle_group": phase["cycle_group"],
+                       "bfs_trees_per_launch": phase["bfs_group"],
                        "walk": "two-ended" if args.walk == 0 else "alg3-descent",
                        "avg_cycle_len": per_tree_sumk / max(1, c_nt),
                        "max_depth": phase["max_depth"],
@@ -378,14 +450,18 @@ def main():
                              else "graph fits L2; consecutive steps use new seeds (new trees)",
                        "parallelism": f"trees t mod {world}; NCCL all-reduce of counters" if world > 1
                                       else "1 GPU"},
-            "gpu_launches": launches,
+            "gpu_launches": launches_per_step * args.steps,
+            "steps_detail": steps_summary,
             "phase_ms_per_step": {k: v for k, v in ph.items()},
+            "graphb_only_ms_per_tree": graphb_only,
             "roofline": roofline,
             "cpu_baseline": cpu,
             "e2e": e2e,
             "clocks": clocks,
         }
         print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
     graphb.free()
     if world > 1:
         dist.destroy_process_group()

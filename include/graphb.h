@@ -135,7 +135,8 @@ int gb_set_option(const char *key, int64_t value);
  * ints[0] trees, [1] sum of cycle lengths, [2] cycles, [3] kernel launches,
  * [4] batches, [5] max tree depth, [6] batch size used, [7] cycle group used,
  * [8] edges of some Sigma_T that contradict the L224 bipartition (option
- * "harary" only; 0 means every balanced state was checked and consistent).
+ * "harary" only; 0 means every balanced state was checked and consistent),
+ * [9] trees per labelling launch, [10] trees per BFS launch.
  * phase_ms[GB_NPHASE] (valid when "timing" was 1): summed CUDA-event times.
  * Returns the number of ints written. */
 #define GB_NPHASE 6

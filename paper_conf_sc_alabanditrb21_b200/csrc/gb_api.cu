@@ -58,10 +58,14 @@ struct Options {
     int64_t wilson = 0;      // sampler 1: 0 one thread per tree (W trees at once), 1 parallel cycle popping
     int64_t harary = 0;      // 1: Harary sides by the L224 procedure (gb_harary.cu)
     int64_t jump = 1;        // walk 0: levels per ancestor record of the cycle walk (1, 2, 4)
+    int64_t bfs = 1;         // 1 multi-source BFS (gb_msbfs.cu, default), 0 tree-parallel pull BFS (gb_tbfs.cu)
+    int64_t bfs_group = 4;   // bfs 0: trees per BFS launch (1..kTbMax)
+    int64_t push_k = 4;      // bfs 0: a level pushes while frontier slots * push_k < unvisited slots
 };
 
 struct Stats {
     int64_t trees = 0, launches = 0, batches = 0, batch_used = 0, group_used = 0, harary_bad = 0;
+    int64_t sub_used = 0, bfs_group_used = 0;   // trees per labelling launch / per BFS launch
     uint64_t sumk = 0, cycles = 0;
     int64_t max_depth = 0;
     double phase_ms[GB_NPHASE] = {0};
@@ -105,13 +109,21 @@ static void free_ws(Workspace &w) {
                     w.parq, w.offq, w.szq, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
                     w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof,
-                    w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey};
+                    w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey, w.tbm, w.tbhbest, w.tbhpos, w.tbhlev};
     for (void *p : ptrs) if (p) cudaFree(p);
     w = Workspace();
 }
 
 static void free_graph(Graph &g) {
     g = Graph();   // the arrays live in the persistent arena
+}
+
+static BfsOpts bfs_opts() {
+    BfsOpts b;
+    b.kind = (int)S.opt.bfs;
+    b.group = (int)S.opt.bfs_group;
+    b.push_k = (int)S.opt.push_k;
+    return b;
 }
 
 static size_t per_tree_bytes(const Graph &g, bool descent) {
@@ -152,6 +164,21 @@ static int ensure_workspace(int B, bool descent) {
     ALLOC(w.msflag, 8);
     ALLOC(w.mscnt, (int64_t)kMsBatch * 2048);
     ALLOC(w.fbm, 6 * ((n + 31) / 32));
+    {   // tree-parallel BFS: bitmaps and hub tables of kTbMax trees
+        const int64_t G = kTbMax, nh = std::max<int64_t>(g.nmulti, 1);
+        ALLOC(w.tbm, (G * 6 + 1) * ((n + 31) / 32));
+        ALLOC(w.tbhbest, G * nh);
+        ALLOC(w.tbhpos, G * nh);
+        ALLOC(w.tbhlev, G * nh);
+        if (cudaMemset(w.tbhbest, 0xFF, sizeof(unsigned long long) * G * nh) != cudaSuccess ||
+            cudaMemset(w.tbhpos, 0xFF, sizeof(uint32_t) * G * nh) != cudaSuccess ||
+            cudaMemset(w.tbhlev, 0, sizeof(uint32_t) * G * nh) != cudaSuccess) {
+            set_error("memset (tbfs hub tables) failed");
+            free_ws(S.ws);
+            return GB_ECUDA;
+        }
+        w.tbg = kTbMax;
+    }
     ALLOC(w.qv, Bn);
     ALLOC(w.lvl, (int64_t)B * (n + 2));
     ALLOC(w.vbase, (int64_t)B * (n + 2));
@@ -176,7 +203,7 @@ static int ensure_workspace(int B, bool descent) {
         w.scan_tmp_elems = scan_tmp_elems(Bn);
         ALLOC(w.scan_tmp, (int64_t)w.scan_tmp_elems);
     } else {
-        ALLOC(w.size, Bn);
+        ALLOC(w.size, (int64_t)B * size_slots(n));
     }
     w.B = B;
     w.n = n;
@@ -349,6 +376,8 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     if (S.ws.msprof) GB_CUDA_TRY(cudaMemsetAsync(S.ws.msprof, 0, sizeof(unsigned long long) * 2048, st));
     T.batch_used = B;
     T.group_used = G;
+    T.sub_used = auto_sub(B);
+    T.bfs_group_used = S.opt.sampler != 0 ? 1 : S.opt.bfs == 1 ? B : std::min<int64_t>(B, S.opt.bfs_group);
     std::vector<cudaEvent_t> &evs = T.evs;
     const bool timing = S.opt.timing != 0;
     int64_t done = 0;
@@ -399,7 +428,8 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
             given = reinterpret_cast<const int32_t *>(S.ws.wseq) + j * S.g.n;
         }
         rc = run_batch_tree(S.g, S.ws, nb, given, st, &T.launches, ev, descent, auto_sub(nb),
-                            (int)S.opt.recpass, (size_t)S.opt.persist, given ? 0 : (int)S.opt.sampler);
+                            (int)S.opt.recpass, (size_t)S.opt.persist, given ? 0 : (int)S.opt.sampler,
+                            bfs_opts());
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
         rc = run_batch_cycles(S.g, S.ws, nb, G, descent, st, &T.launches, jump);
@@ -455,7 +485,7 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
         d_given = reinterpret_cast<const int32_t *>(S.ws.wseq);
     }
     rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk == 1, 1,
-                        0, 0, d_given ? 0 : (int)S.opt.sampler);
+                        0, 0, d_given ? 0 : (int)S.opt.sampler, bfs_opts());
     if (rc) return rc;
     if (user_tree) {
         unsigned long long vis = 0;
@@ -625,6 +655,18 @@ int gb_set_option(const char *key, int64_t value) {
         S.opt.sampler = value;
     }
     else if (!strcmp(key, "recpass")) S.opt.recpass = value != 0;
+    else if (!strcmp(key, "bfs")) {
+        if (value != 0 && value != 1) { set_error("bfs must be 0 (tree-parallel) or 1 (multi-source)"); return GB_EINVAL; }
+        S.opt.bfs = value;
+    }
+    else if (!strcmp(key, "bfs_group")) {
+        if (value < 1 || value > kTbMax) { set_error("bfs_group must be 1..16"); return GB_EINVAL; }
+        S.opt.bfs_group = value;
+    }
+    else if (!strcmp(key, "push_k")) {
+        if (value < 0 || value > 1024) { set_error("push_k must be 0..1024"); return GB_EINVAL; }
+        S.opt.push_k = value;
+    }
     else if (!strcmp(key, "jump")) {
         if (value != 1 && value != 2 && value != 4) { set_error("jump must be 1, 2 or 4"); return GB_EINVAL; }
         S.opt.jump = value;
@@ -686,21 +728,17 @@ int gb_tree_debug(int64_t t, uint64_t seed, int32_t *parent, int32_t *dist, int3
     if (rc) return rc;
     const int64_t n = S.g.n;
     int32_t *d_tmp = nullptr;
-    GB_CUDA_TRY(cudaMalloc(&d_tmp, sizeof(int32_t) * 3 * n));
-    rc = debug_tree_views(S.g, S.ws, S.opt.walk == 1, d_tmp, d_tmp + n, d_tmp + 2 * n, S.stream);
+    GB_CUDA_TRY(cudaMalloc(&d_tmp, sizeof(int32_t) * 4 * n));
+    rc = debug_tree_views(S.g, S.ws, S.opt.walk == 1, d_tmp, d_tmp + n, d_tmp + 2 * n, d_tmp + 3 * n, S.stream);
     if (rc) { cudaFree(d_tmp); return rc; }
-    std::vector<int32_t> h(3 * n);
-    cudaError_t ce = cudaMemcpy(h.data(), d_tmp, sizeof(int32_t) * 3 * n, cudaMemcpyDeviceToHost);
+    std::vector<int32_t> h(4 * n);
+    cudaError_t ce = cudaMemcpy(h.data(), d_tmp, sizeof(int32_t) * 4 * n, cudaMemcpyDeviceToHost);
     cudaFree(d_tmp);
     GB_CUDA_TRY(ce);
     if (parent) std::copy(h.begin(), h.begin() + n, parent);
     if (dist) std::copy(h.begin() + n, h.begin() + 2 * n, dist);
-    if (size) std::copy(h.begin() + 2 * n, h.end(), size);
-    if (pre) {
-        std::vector<uint32_t> tmp(n);
-        GB_CUDA_TRY(cudaMemcpy(tmp.data(), S.ws.pp, 4 * n, cudaMemcpyDeviceToHost));
-        for (int64_t v = 0; v < n; v++) pre[v] = (int32_t)(tmp[v] & kIdMask);
-    }
+    if (size) std::copy(h.begin() + 2 * n, h.begin() + 3 * n, size);
+    if (pre) std::copy(h.begin() + 3 * n, h.end(), pre);
     if (flip) { rc = copy_flips(flip); if (rc) return rc; }
     return copy_cycle_stats(sum_cycle_len, num_cycles);
 }
@@ -735,10 +773,10 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip, uint64_t *sum_cy
 int gb_get_stats(int64_t *ints, int n_ints, double *phase_ms, int n_phase) {
     if (finalize_stats()) return GB_ECUDA;
     const Stats &T = S.st;
-    int64_t v[9] = {T.trees, (int64_t)T.sumk, (int64_t)T.cycles, T.launches, T.batches,
-                    T.max_depth, T.batch_used, T.group_used, T.harary_bad};
+    int64_t v[11] = {T.trees, (int64_t)T.sumk, (int64_t)T.cycles, T.launches, T.batches,
+                     T.max_depth, T.batch_used, T.group_used, T.harary_bad, T.sub_used, T.bfs_group_used};
     int k = 0;
-    for (; ints && k < n_ints && k < 9; k++) ints[k] = v[k];
+    for (; ints && k < n_ints && k < 11; k++) ints[k] = v[k];
     for (int i = 0; phase_ms && i < n_phase && i < GB_NPHASE; i++) phase_ms[i] = T.phase_ms[i];
     return k;
 }

@@ -30,7 +30,7 @@
 namespace gb {
 
 struct CycleParams {
-    const uint2 *edges;
+    const uint2 *edges;    // [m] {u, v | neg<<31} by eid, internal ids (the labels' index space)
     int64_t n, m;
     const uint32_t *pp;    // [B][n] pre | pi<<31
     const uint2 *rec;      // [B][n] pre-indexed {up | neg<<31, size}
@@ -349,12 +349,14 @@ __global__ void k_accumulate_edges(const uint32_t *__restrict__ fbits, int64_t w
     }
 }
 
+// (labels in internal ids i; the counter of the original vertex bord[i])
 __global__ void k_accumulate_agree(const uint32_t *__restrict__ pp, const uint32_t *__restrict__ s1,
-                                   const int32_t *__restrict__ comp, const int32_t *__restrict__ coff,
+                                   const int32_t *__restrict__ comp_i, const int32_t *__restrict__ coff,
+                                   const uint32_t *__restrict__ bord,
                                    int64_t n, int64_t ncomp, int B, int32_t *__restrict__ agree) {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
          v += (int64_t)gridDim.x * blockDim.x) {
-        const int32_t C = __ldg(comp + v);
+        const int32_t C = __ldg(comp_i + v);
         const uint32_t cs = (uint32_t)(__ldg(coff + C + 1) - __ldg(coff + C));
         int32_t d = 0;
         for (int b = 0; b < B; b++) {
@@ -363,7 +365,7 @@ __global__ void k_accumulate_agree(const uint32_t *__restrict__ pp, const uint32
             const uint32_t other = cs - mine;
             d += mine > other ? 2 : (mine == other ? 1 : 0);
         }
-        agree[v] += d;
+        agree[__ldg(bord + v)] += d;
     }
 }
 
@@ -378,7 +380,7 @@ int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool desce
     CycleParams P;
     if (descent || !ws.jrec) jump = 1;
     P.jrec = ws.jrec;
-    P.edges = g.edges; P.n = g.n; P.m = g.m;
+    P.edges = g.edges_i; P.n = g.n; P.m = g.m;
     P.pp = ws.pp; P.rec = ws.rec; P.crec = ws.crec; P.clist = ws.clist;
     P.fbits = ws.fbits; P.tstat = ws.tstat;
     P.words = (g.m + 31) / 32;
@@ -412,7 +414,7 @@ int run_batch_accumulate(const Graph &g, Workspace &ws, int B, int32_t *d_cnt, i
         ++*launches;
     }
     k_accumulate_agree<<<grid_cap(g.n, 256, g.num_sms, 16), 256, 0, st>>>(
-        ws.pp, ws.s1, g.comp, g.coff, g.n, g.ncomp, B, d_agree);
+        ws.pp, ws.s1, g.comp_i, g.coff, g.bord, g.n, g.ncomp, B, d_agree);
     ++*launches;
     GB_CUDA_TRY(cudaGetLastError());
     return GB_OK;

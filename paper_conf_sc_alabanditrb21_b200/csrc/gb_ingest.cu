@@ -325,6 +325,25 @@ __global__ void k_item_fill(const uint32_t *__restrict__ brow, const uint32_t *_
 // ---------------------------------------------------------------------------
 // Degree-sorted view for the multi-source BFS (gb_msbfs.cu)
 // ---------------------------------------------------------------------------
+// the edge table and the component ranks in internal ids (the tree pipeline's
+// index space: hubs first, so the parents -- mostly high-degree vertices --
+// cluster at the front of every per-tree label array)
+__global__ void k_internal_edges(const uint2 *__restrict__ edges, const uint32_t *__restrict__ brank,
+                                 int64_t m, uint2 *__restrict__ edges_i) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        const uint2 ed = edges[e];
+        edges_i[e] = make_uint2(brank[ed.x], brank[ed.y & kIdMask] | (ed.y & kNegBit));
+    }
+}
+
+__global__ void k_internal_comp(const int32_t *__restrict__ comp, const uint32_t *__restrict__ bord,
+                                int64_t n, int32_t *__restrict__ comp_i) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x)
+        comp_i[i] = comp[bord[i]];
+}
+
 __global__ void k_degrees(const uint32_t *__restrict__ rp, int64_t n, uint32_t *__restrict__ deg,
                           uint32_t *__restrict__ ids) {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
@@ -559,6 +578,14 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
             k_item_fill<<<grid_for(g.nlight0, 256, sms), 256, 0, st>>>(g.brow, uptr, g.nlight0, g.items);
             ++*launches;
         }
+        ING_ALLOC(g.edges_i, kArEdgesI, m);
+        ING_ALLOC(g.comp_i, kArCompI, n);
+        if (m) {
+            k_internal_edges<<<grid_for(m, 256, sms), 256, 0, st>>>(g.edges, g.brank, m, g.edges_i);
+            ++*launches;
+        }
+        k_internal_comp<<<grid_for(n, 256, sms), 256, 0, st>>>(g.comp, g.bord, n, g.comp_i);
+        ++*launches;
         ING_TRY(cudaStreamSynchronize(st));
     }
     g.n = n;

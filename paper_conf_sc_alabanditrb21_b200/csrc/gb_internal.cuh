@@ -18,6 +18,7 @@ constexpr int kBlock = 256;                  // threads per CTA of the cooperati
 constexpr int kMsBatch = 64;                 // trees per multi-source BFS (one bit each)
 constexpr int kLight = 8;                    // BFS: degree <= kLight -> one lane per vertex
 constexpr int kChunk = 256;                  // BFS: slots per warp work item of a heavier vertex
+constexpr int kTbMax = 16;                   // tree-parallel BFS: trees per launch (per-tree bitmaps)
 
 // ---------------------------------------------------------------------------
 // Counter-based hash: SplitMix64 finaliser and its inverse (R4).
@@ -111,7 +112,11 @@ struct Graph {
     uint32_t *row_ptr = nullptr;        // [n+1]
     uint32_t *adj = nullptr;            // [2m] col | neg<<31
     uint32_t *adj_eid = nullptr;        // [2m] eid of the slot
-    uint2 *edges = nullptr;             // [m] {u, v | neg<<31}, u < v, index = eid
+    uint2 *edges = nullptr;             // [m] {u, v | neg<<31}, u < v, index = eid (original ids)
+    // The tree pipeline (level lists, Alg. 4 labels, the cycle walk, the agree
+    // accumulation) runs on the internal ids of the degree-sorted view below:
+    uint2 *edges_i = nullptr;           // [m] {brank u, brank v | neg<<31}, index = eid
+    int32_t *comp_i = nullptr;          // [n] component rank of internal vertex i
     int32_t *comp = nullptr;            // [n] component rank (by minimum vertex)
     int32_t *coff = nullptr;            // [ncomp+1] component offsets (pre of the root)
     int32_t *cverts = nullptr;          // [n] vertices grouped by component, ascending
@@ -174,6 +179,12 @@ struct Workspace {
                                         // [4..6] frontier sizes (levels mod 3)
     uint32_t *mscnt = nullptr;          // [64][2048] per-block discovery counts
     unsigned long long *msprof = nullptr;  // [256][4] BFS phase timestamps (option "msprof")
+    // tree-parallel BFS state (gb_tbfs.cu), G <= kTbMax trees per launch
+    uint32_t *tbm = nullptr;            // [G][6][ceil(n/32)] per-tree bitmaps + [ceil(n/32)] "finished"
+    unsigned long long *tbhbest = nullptr; // [G][nmulti] hub parent keys
+    uint32_t *tbhpos = nullptr;         // [G][nmulti] hub list positions
+    uint32_t *tbhlev = nullptr;         // [G][nmulti] hub discovery level + 2
+    int tbg = 0;                        // G the buffers hold
     uint32_t *fbm = nullptr;            // [6][ceil(n/32)] frontier bitmaps (3), finished bitmap,
                                         // two push bitmaps (direction optimisation)
     uint32_t *s1 = nullptr;    // [B][ncomp] #vertices with pi = 1 per component
@@ -190,6 +201,13 @@ struct Workspace {
     uint32_t *scan_tmp = nullptr;
     size_t scan_tmp_elems = 0;
 };
+
+// subtree-size counters per tree (walk 0): the power of two >= n (gb_tree.cu szi)
+inline int64_t size_slots(int64_t n) {
+    int64_t s = 2;
+    while (s < n) s <<= 1;
+    return s;
+}
 
 struct BatchArgs {
     int B;                 // trees in this batch
@@ -221,7 +239,7 @@ enum ArenaSlot {
     kArRowPtr64, kArCol, kArSign, kArErr, kArRowPtr, kArAdj, kArAdjEid, kArEdges, kArComp,
     kArCverts, kArUptr, kArUpc, kArEbase, kArScanTmp, kArLab, kArFlag, kArRank, kArCoff,
     kArBrow, kArBadj, kArBorig, kArBord, kArBrank, kArItems, kArDeg, kArSortTmp, kArCkeys,
-    kArSlots
+    kArEdgesI, kArCompI, kArSlots
 };
 void *arena(int slot, size_t bytes);   // nullptr on allocation failure (error set)
 void arena_free_all();
@@ -233,9 +251,15 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr,
            const int32_t *h_col, const int8_t *h_sign, cudaStream_t st,
            int64_t *launches);
 
+struct BfsOpts {
+    int kind = 1;     // 1 multi-source BFS (gb_msbfs.cu), 0 tree-parallel pull BFS (gb_tbfs.cu)
+    int group = 4;    // kind 0: trees per launch
+    int push_k = 4;   // kind 0: a level pushes while frontier slots * push_k < unvisited slots
+};
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
                    cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub,
-                   int recpass = 0, size_t persist = 0, int sampler = 0);
+                   int recpass = 0, size_t persist = 0, int sampler = 0,
+                   const BfsOpts &bfs = BfsOpts());
 
 // f.3: uniform random spanning forest of tree ws.tkey[0] (Wilson by parallel
 // cycle popping, gb_wilson.cu) -> parent (-1 at the roots)
@@ -259,9 +283,12 @@ struct MsBfsOut {
 };
 int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStream_t st,
               int64_t *launches);
+// tree-parallel pull BFS (gb_tbfs.cu): the same outputs, G trees per launch
+int run_tbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStream_t st,
+             int64_t *launches, int G, int push_k);
 
 int debug_tree_views(const Graph &g, Workspace &ws, bool descent, int32_t *d_parent,
-                     int32_t *d_dist, int32_t *d_size, cudaStream_t st);
+                     int32_t *d_dist, int32_t *d_size, int32_t *d_pre, cudaStream_t st);
 
 int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool descent,
                      cudaStream_t st, int64_t *launches, int jump = 1);

@@ -18,8 +18,10 @@
 // one read of w's adjacency serving all B trees.  For every tree t in new(w)
 // the parent of w is the neighbour u with bit t in F_L[u] (one level up)
 // minimising parent_key(t, u, w) (reading R4).  Discoveries go to the
-// per-tree level lists (qv, parq: original ids, the layout the labelling
-// passes stream).
+// per-tree level lists (qv, parq) as internal ids: the labelling passes and
+// the cycle walk index their per-tree arrays by the degree-sorted ids, so the
+// parents -- mostly hubs and other high-degree vertices -- share a small hot
+// region of each array.
 //
 // Work mapping (degree-sorted internal ids, gb_ingest.cu):
 //   light vertices (degree <= kLight): one lane per vertex;
@@ -102,19 +104,22 @@ __device__ __forceinline__ unsigned long long fr_word(const unsigned long long *
     return bm_test(bm, u) ? __ldcg(F + u) : 0ull;
 }
 
-// level-(L+1) entry `pos` of tree t: the vertex and its parent | neg << 31
-__device__ __forceinline__ void ms_emit(const MsParams &P, int t, uint32_t pos, uint32_t ow,
+// level-(L+1) entry `pos` of tree t: the vertex and its parent | neg << 31,
+// both as internal (degree-sorted) ids -- the index space of the labelling
+// passes and the walk.  Keys and `par` carry the parent's original id (the
+// min-hash rule R4 is defined on original ids), translated here.
+__device__ __forceinline__ void ms_emit(const MsParams &P, int t, uint32_t pos, uint32_t vi,
                                         unsigned long long key) {
     const size_t o = (size_t)t * P.n + pos;
-    P.qv[o] = ow;
-    P.parq[o] = ((uint32_t)(key >> 1) & kIdMask) | ((uint32_t)key << 31);
+    P.qv[o] = vi;
+    P.parq[o] = __ldg(P.brank + ((uint32_t)(key >> 1) & kIdMask)) | ((uint32_t)key << 31);
 }
 
-__device__ __forceinline__ void ms_emit_par(const MsParams &P, int t, uint32_t pos, uint32_t ow,
+__device__ __forceinline__ void ms_emit_par(const MsParams &P, int t, uint32_t pos, uint32_t vi,
                                             uint32_t par) {
     const size_t o = (size_t)t * P.n + pos;
-    P.qv[o] = ow;
-    P.parq[o] = par;
+    P.qv[o] = vi;
+    P.parq[o] = __ldg(P.brank + (par & kIdMask)) | (par & kNegBit);
 }
 
 // OR of the frontier words over the slots [s0, s1) (one warp, lanes stride)
@@ -186,8 +191,9 @@ __device__ __forceinline__ void ms_chunk_keys(const MsParams &P, const unsigned 
 constexpr int kMultiCap = 512;           // multi-candidate pairs per round
 struct WarpScratch {
     uint32_t ml[kMultiCap];              // multi-candidate pairs: src << 14 | tree << 8 | slot mask
-    uint8_t sidx[kMsBatch][32];          // single-candidate slot of (tree, lane)
-    uint32_t lo[kLight][32];             // candidate neighbour (original id) | neg << 31
+    unsigned long long pk[3][32];        // parent slot index k of (vertex lane, tree), bit-planes
+    uint32_t lo[kLight][32];             // candidate neighbour (original id) | neg << 31 (hashing)
+    uint32_t li[kLight][32];             // the same neighbour as an internal id | neg << 31 (output)
     uint32_t ow[32];                     // original id of each lane's vertex
     unsigned long long best[kMsBatch];   // item parents: best key per tree
 };
@@ -197,13 +203,32 @@ __device__ __forceinline__ uint32_t key_to_par(unsigned long long key) {
     return ((uint32_t)(key >> 1) & kIdMask) | ((uint32_t)key << 31);
 }
 
+// 32 x 32 bit-matrix transpose across the warp: lane r holds row r (bit c =
+// M[r][c]); afterwards lane c holds column c (bit r = M[r][c]).  Five rounds
+// of off-diagonal block swaps.
+__device__ __forceinline__ uint32_t transpose32(uint32_t x) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int sh = 16; sh; sh >>= 1) {
+        const uint32_t m = sh == 16 ? 0x0000FFFFu : sh == 8 ? 0x00FF00FFu : sh == 4 ? 0x0F0F0F0Fu
+                         : sh == 2 ? 0x33333333u : 0x55555555u;
+        const uint32_t y = __shfl_xor_sync(0xFFFFFFFFu, x, sh);
+        x = (lane & sh) ? ((x & ~m) | ((y & ~m) >> sh)) : ((x & m) | ((y & m) << sh));
+    }
+    return x;
+}
+
 // parents of the light vertices queued by a warp (lane l: internal id i,
 // valid if `act`) in the trees each discovered on this level (F_{L+1}[i]).
-// Trees in which a vertex has a single candidate (one neighbour one level
-// up) take it: the warp walks those trees, the lanes concerned take
-// consecutive positions of the tree's level list (coalesced writes).  The
-// (vertex, tree) pairs with several candidates are listed and hashed one per
-// lane (the min-hash rule, reading R4).
+// Per lane, c[k] = the trees in which neighbour k is one level up.  A tree
+// with a single candidate takes it: its slot index k goes into three
+// bit-planes (pk[j] bit t = bit j of k) with three ORs per neighbour, no
+// per-tree loop.  The (vertex, tree) pairs with several candidates are listed
+// and hashed one per lane (the min-hash rule, reading R4); the winner's k is
+// OR-ed into the planes.  Emission is transposed: the warp's 32 discovery
+// words (vertex x tree bits) are transposed so that lane t holds, for trees
+// t and t + 32, the mask of vertices to append; it reserves its run of the
+// tree's level list with one shared-memory add and writes its entries.
 __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsigned long long *F,
                                                  const unsigned long long *Nx, const uint32_t *bm,
                                                  uint32_t i, bool act, const uint64_t *s_tk,
@@ -224,20 +249,35 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
             if (k < (int)deg) {
                 const uint32_t a = __ldg(P.badj + rs + k);
                 c[k] = fr_word(F, bm, a & kIdMask) & nw;
-                if (c[k]) W.lo[k][lane] = __ldg(P.borig + rs + k) | (a & kNegBit);
+                if (c[k]) {
+                    W.lo[k][lane] = __ldg(P.borig + rs + k) | (a & kNegBit);
+                    W.li[k][lane] = a;
+                }
                 s2m |= s1m & c[k];
                 s1m |= c[k];
             }
         }
-#pragma unroll
-        for (int k = 0; k < kLight; k++)
-            for (unsigned long long m = c[k] & ~s2m; m; m &= m - 1) W.sidx[__ffsll((long long)m) - 1][lane] = (uint8_t)k;
     } else {
 #pragma unroll
         for (int k = 0; k < kLight; k++) c[k] = 0;
     }
     W.ow[lane] = ow;
-    // several candidates: listed pairs, hashed one per lane
+    {   // slot-index planes of the single-candidate trees
+        const unsigned long long sm = ~s2m;
+        unsigned long long p0 = 0, p1 = 0, p2 = 0;
+#pragma unroll
+        for (int k = 0; k < kLight; k++) {
+            const unsigned long long ck = c[k] & sm;
+            if (k & 1) p0 |= ck;
+            if (k & 2) p1 |= ck;
+            if (k & 4) p2 |= ck;
+        }
+        W.pk[0][lane] = p0;
+        W.pk[1][lane] = p1;
+        W.pk[2][lane] = p2;
+    }
+    // several candidates: listed pairs, hashed one per lane; the winning slot
+    // index goes into the planes
     const uint32_t cnt = (uint32_t)__popcll(s2m);
     const uint32_t incl = warp_incl_scan32(cnt);
     const uint32_t total = __shfl_sync(0xFFFFFFFFu, incl, 31);
@@ -263,26 +303,47 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
             const uint32_t o_w = W.ow[src];
             const uint64_t tk = s_tk[t];
             unsigned long long best = ~0ull;
+            uint32_t bk = 0;
             for (uint32_t km = e & 0xFFu; km; km &= km - 1) {
-                const uint32_t o = W.lo[__ffs(km) - 1][src];
-                best = min(best, parent_key(tk, o & kIdMask, o_w, o >> 31));
+                const uint32_t k = __ffs(km) - 1;
+                const uint32_t o = W.lo[k][src];
+                const unsigned long long key = parent_key(tk, o & kIdMask, o_w, o >> 31);
+                if (key < best) { best = key; bk = k; }
             }
-            ms_emit(P, t, s_base[t] + atomicAdd(&s_pos[t], 1u), o_w, best);
+            const unsigned long long bit = 1ull << t;
+            if (bk & 1) atomicOr(&W.pk[0][src], bit);
+            if (bk & 2) atomicOr(&W.pk[1][src], bit);
+            if (bk & 4) atomicOr(&W.pk[2][src], bit);
         }
         __syncwarp();
     }
-    // single candidate: no hash; tree by tree, coalesced
-    const unsigned long long sm = nw & ~s2m;
+    __syncwarp();   // planes of every lane complete
+    // emission: one shared-memory reservation per tree (lane t reserves the
+    // runs of trees t and t + 32, sized by the transposed discovery words),
+    // then tree by tree the discovering lanes write consecutive entries of the
+    // tree's level list (coalesced); the parent slot k comes from the planes
+    const unsigned long long mine_pk0 = W.pk[0][lane], mine_pk1 = W.pk[1][lane], mine_pk2 = W.pk[2][lane];
+    const uint32_t nlo = transpose32((uint32_t)nw);
+    const uint32_t nhi = transpose32((uint32_t)(nw >> 32));
+    uint32_t blo = 0, bhi = 0;
+    if (nlo) blo = s_base[lane] + atomicAdd(&s_pos[lane], (uint32_t)__popc(nlo));
+    if (nhi) bhi = s_base[lane + 32] + atomicAdd(&s_pos[lane + 32], (uint32_t)__popc(nhi));
     const uint32_t lt = (1u << lane) - 1u;
-    for (unsigned long long rem = warp_or64(sm); rem; rem &= rem - 1) {
-        const int t = __ffsll((long long)rem) - 1;
-        const bool has = (sm >> t) & 1ull;
-        const uint32_t mask = __ballot_sync(0xFFFFFFFFu, has);
-        const int leader = __ffs(mask) - 1;
-        uint32_t b = 0;
-        if (lane == leader) b = atomicAdd(&s_pos[t], (uint32_t)__popc(mask));
-        b = __shfl_sync(0xFFFFFFFFu, b, leader);
-        if (has) ms_emit_par(P, t, s_base[t] + b + (uint32_t)__popc(mask & lt), ow, W.lo[W.sidx[t][lane]][lane]);
+#pragma unroll
+    for (int h = 0; h < 2; h++) {
+        for (uint32_t trees = __ballot_sync(0xFFFFFFFFu, (h ? nhi : nlo) != 0); trees; trees &= trees - 1) {
+            const int tl = __ffs(trees) - 1;
+            const int t = tl + 32 * h;
+            const uint32_t mask = __shfl_sync(0xFFFFFFFFu, h ? nhi : nlo, tl);
+            const uint32_t base = __shfl_sync(0xFFFFFFFFu, h ? bhi : blo, tl);
+            if ((mask >> lane) & 1u) {
+                const uint32_t k = (uint32_t)((mine_pk0 >> t) & 1ull) | ((uint32_t)((mine_pk1 >> t) & 1ull) << 1) |
+                                   ((uint32_t)((mine_pk2 >> t) & 1ull) << 2);
+                const size_t o = (size_t)t * P.n + base + __popc(mask & lt);
+                P.qv[o] = i;
+                P.parq[o] = W.li[k][lane];
+            }
+        }
     }
     __syncwarp();
 }
@@ -381,15 +442,15 @@ __global__ void k_ms_roots(MsParams P) {
         if (P.brow[ri + 1] == P.brow[ri]) {
             // isolated vertex: a one-vertex tree, finished here (pi = 0)
             const uint32_t pre = (uint32_t)P.coff[C];
-            P.pp[nb + r] = pre;
+            P.pp[nb + ri] = pre;
             P.rec[nb + pre] = make_uint2(pre, 1u);
             if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
             continue;
         }
         const unsigned long long old = atomicAdd((unsigned long long *)(P.lvl + b * P.ls), 1ull << 32);
         const uint32_t pos = (uint32_t)(old >> 32);
-        P.qv[nb + pos] = r;
-        P.parq[nb + pos] = r;
+        P.qv[nb + pos] = ri;
+        P.parq[nb + pos] = ri;
         atomicOr(P.fr + ri, bit);
         atomicOr(P.fbm + (ri >> 5), 1u << (ri & 31));
     }
@@ -547,13 +608,19 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                         P.vis[i] = vis | nw;
                         Nx[i] = nw;
                         nowfull = (vis | nw) == full;
-                        for (unsigned long long r = nw; r; r &= r - 1)
-                            atomicAdd(&s_cnt[__ffsll((long long)r) - 1], 1u);
                     } else {
                         nowfull = vis == full;
                     }
                 }
                 const uint32_t fb = __ballot_sync(0xFFFFFFFFu, nw != 0);
+                if (fb) {
+                    // per-tree discovery counts: transpose the warp's 32 words
+                    // so that lane t counts tree t (and t + 32)
+                    const uint32_t clo = __popc(transpose32((uint32_t)nw));
+                    const uint32_t chi = __popc(transpose32((uint32_t)(nw >> 32)));
+                    if (clo) atomicAdd(&s_cnt[lane], clo);
+                    if (chi) atomicAdd(&s_cnt[lane + 32], chi);
+                }
                 const uint32_t nf = __ballot_sync(0xFFFFFFFFu, nowfull);
                 if (lane == 0 && fb) atomicAdd(&s_fc, (uint32_t)__popc(fb));
                 if (lane == 0 && nf) atomicAdd(&s_ff, (uint32_t)__popc(nf));
@@ -629,9 +696,9 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                         p1 = key_to_par(b1);
                     }
                     if ((nw >> lane) & 1ull)
-                        ms_emit_par(P, lane, s_base[lane] + atomicAdd(&s_pos[lane], 1u), ow, p0);
+                        ms_emit_par(P, lane, s_base[lane] + atomicAdd(&s_pos[lane], 1u), i, p0);
                     if ((nw >> (lane + 32)) & 1ull)
-                        ms_emit_par(P, lane + 32, s_base[lane + 32] + atomicAdd(&s_pos[lane + 32], 1u), ow, p1);
+                        ms_emit_par(P, lane + 32, s_base[lane + 32] + atomicAdd(&s_pos[lane + 32], 1u), i, p1);
                 }
             } else {
                 // light vertices: the warp queues its discovered vertices and
@@ -682,7 +749,6 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
             for (int64_t hi = gwarp; hi < P.nmulti; hi += nwarps) {
                 const unsigned long long want = __ldcg(P.hacc + hi);
                 if (!want) continue;
-                const uint32_t ow = __ldg(P.bord + hi);
 #pragma unroll
                 for (int h = 0; h < 2; h++) {
                     const int t = lane + 32 * h;
@@ -692,7 +758,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                         *slot = ~0ull;
                         const unsigned long long old =
                             atomicAdd((unsigned long long *)(P.lvl + t * P.ls + L + 1), 1ull << 32);
-                        ms_emit(P, t, s_vb[t] + (uint32_t)(old >> 32), ow, key);
+                        ms_emit(P, t, s_vb[t] + (uint32_t)(old >> 32), (uint32_t)hi, key);
                     }
                 }
                 __syncwarp();

@@ -34,8 +34,9 @@ namespace gb {
 namespace cg = cooperative_groups;
 
 struct TreeParams {
-    const uint32_t *row_ptr, *adj;
-    const int32_t *comp, *coff, *cverts;
+    const uint32_t *row_ptr, *adj;             // original CSR (push BFS of caller trees)
+    const uint32_t *brank, *bord;              // original <-> internal ids
+    const int32_t *comp, *comp_i, *coff, *cverts;
     int64_t n, ncomp, nw;  // nw = state words per tree ((n + 3) / 4)
     int32_t cbig;
     int B;
@@ -45,7 +46,8 @@ struct TreeParams {
     unsigned long long *pkeyq;
     uint64_t *lvl;
     uint32_t *vbase;
-    uint32_t *size;             // vertex-indexed subtree size (walk 0)
+    uint32_t *size;             // subtree-size counters (walk 0), slot szi(i) of vertex i,
+                                // tree stride szn (see szi)
     unsigned long long *sz64;   // vertex-indexed (children << 32 | size) (walk 1)
     uint32_t *parq, *offq, *szq, *cidxq;
     uint32_t *pp;
@@ -58,9 +60,22 @@ struct TreeParams {
     uint2 *crec;                 // walk 1
     unsigned long long *visited; // [B] vertices reached (given-tree validation)
     unsigned long long *prof;    // option "msprof": [256][4] level timestamps (gb_label_profile)
+    uint32_t szmask;             // szn - 1
+    int64_t szn;                 // size counters per tree (power of two >= n)
     int recpass;                 // walk 0: top-down leaves {up | neg, size} and pre in queue
                                  // order; k_rec_scatter writes rec[pre] afterwards
 };
+
+// Slot of vertex i's subtree-size counter: a multiplicative scramble of the
+// id, i * 0x9E3779B1 mod szn (odd multiplier: a bijection on [0, szn)).
+// Internal ids put the hubs -- the parents of most vertices -- next to each
+// other, and the atomics of the bottom-up pass then queue on a few hot L2
+// sectors; scrambled, a hot counter's sector mates are unrelated (mostly
+// cold) vertices.  (Bit reversal does the same but turns consecutive ids into
+// power-of-two strides: measured slower.)
+__device__ __forceinline__ uint32_t szi(const TreeParams &P, uint32_t i) {
+    return (i * 0x9E3779B1u) & P.szmask;
+}
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
     uint32_t m;
@@ -96,7 +111,9 @@ __global__ void k_batch_prep(TreeParams P) {
     if (b == 0) *P.maxd = 0;
 }
 
-// root of component C in tree b: cverts_C[rkey mod |C|] (reading R4)
+// a root of the caller tree (push BFS of gb_balance_given_tree and the f.3
+// samplers); r is an original id -- the push BFS walks the original CSR, and
+// its level lists are translated to internal ids afterwards (k_pkey_to_parq)
 __device__ __forceinline__ void place_root(const TreeParams &P, int b, int64_t C, uint32_t r) {
     const size_t nb = (size_t)b * P.n;
     atomicOr(P.vst + (size_t)b * P.nw + (r >> 2), level_stamp(0) << (8 * (r & 3)));
@@ -104,7 +121,7 @@ __device__ __forceinline__ void place_root(const TreeParams &P, int b, int64_t C
     const uint32_t pre = (uint32_t)P.coff[C];
     if (deg == 0) {
         // isolated vertex: a one-vertex tree, finished here (pi = 0)
-        P.pp[nb + r] = pre;
+        P.pp[nb + P.brank[r]] = pre;
         P.rec[nb + pre] = make_uint2(pre, 1u);
         if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
         if (P.visited) atomicAdd(P.visited + b, 1ull);
@@ -116,18 +133,6 @@ __device__ __forceinline__ void place_root(const TreeParams &P, int b, int64_t C
     P.qs[nb + pos] = (uint32_t)old;
     P.qr[nb + pos] = P.row_ptr[r];
     P.pkeyq[nb + pos] = ~0ull;
-}
-
-__global__ void k_roots(TreeParams P) {
-    const int64_t total = (int64_t)P.B * P.ncomp;
-    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total;
-         i += (int64_t)gridDim.x * blockDim.x) {
-        const int b = (int)(i / P.ncomp);
-        const int64_t C = i - (int64_t)b * P.ncomp;
-        const uint32_t sz = (uint32_t)(P.coff[C + 1] - P.coff[C]);
-        const uint64_t rk = root_key(P.tkey[b], C);
-        place_root(P, b, C, (uint32_t)P.cverts[P.coff[C] + (int64_t)(rk % sz)]);
-    }
 }
 
 // caller-given tree: its roots (parent == -1); one tree (b = 0)
@@ -531,7 +536,7 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
             constexpr int kILP = GB_ILP_UP;
             GB_QPOL;
             for (unsigned long long base = gtid; base < total; base += kILP * nthr) {
-                size_t qi[kILP], nbk[kILP];
+                size_t qi[kILP], nbk[kILP], sbk[kILP];
                 uint32_t w[kILP], p[kILP], sz[kILP];
                 bool ok[kILP];
 #pragma unroll
@@ -541,6 +546,7 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
                     if (ok[k]) {
                         const int b = tree_of(T, B, i);
                         nbk[k] = (size_t)b * P.n;
+                        sbk[k] = (size_t)b * P.szn;
                         qi[k] = nbk[k] + T.vb[b] + (uint32_t)(i - T.soff[b]);
                         w[k] = GB_QLD(P.qv + qi[k]);
                         p[k] = GB_QLD(P.parq + qi[k]) & kIdMask;
@@ -548,11 +554,11 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
                 }
 #pragma unroll
                 for (int k = 0; k < kILP; k++)
-                    if (ok[k]) sz[k] = 1 + __ldcg(P.size + nbk[k] + w[k]);
+                    if (ok[k]) sz[k] = 1 + __ldcg(P.size + sbk[k] + szi(P, w[k]));
 #pragma unroll
                 for (int k = 0; k < kILP; k++) {
                     if (ok[k]) {
-                        const uint32_t o = atomicAdd(P.size + nbk[k] + p[k], sz[k]);
+                        const uint32_t o = atomicAdd(P.size + sbk[k] + szi(P, p[k]), sz[k]);
                         GB_QST(P.offq + qi[k], 1 + o);
                         GB_QST(P.szq + qi[k], sz[k]);
                     }
@@ -563,18 +569,20 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
              wb += (unsigned long long)nwarps * 32) {
             const unsigned long long i = wb + lane;
             const bool valid = i < total;
-            size_t nb = 0, qi = 0;
+            size_t nb = 0, qi = 0, sb = 0;
             uint32_t w = 0, p = 0, sz = 0, neg = 0;
             if (valid) {
                 const int b = tree_of(T, B, i);
                 nb = (size_t)b * P.n;
+                sb = (size_t)b * P.szn;
                 qi = nb + T.vb[b] + (uint32_t)(i - T.soff[b]);
                 w = __ldcg(P.qv + qi);
                 const uint32_t pq = __ldcg(P.parq + qi);
                 p = pq & kIdMask;
                 neg = pq & kNegBit;
                 // counters hold the sum of the children's sizes: size = 1 + that
-                sz = 1 + (kDescent ? (uint32_t)__ldcg(P.sz64 + nb + w) : __ldcg(P.size + nb + w));
+                sz = 1 + (kDescent ? (uint32_t)__ldcg(P.sz64 + nb + w)
+                                   : __ldcg(P.size + sb + szi(P, w)));
             }
             if (kDescent) {
                 const unsigned long long o =
@@ -584,7 +592,7 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
                     P.cidxq[qi] = (uint32_t)(o >> 32);
                 }
             } else {
-                const uint32_t o = aggregated_add<uint32_t>(P.size + nb + p, sz, valid);
+                const uint32_t o = aggregated_add<uint32_t>(P.size + sb + szi(P, p), sz, valid);
                 if (valid) P.offq[qi] = 1 + o;
             }
             if (valid) P.szq[qi] = sz;
@@ -675,7 +683,7 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
                         P.rec[nbk[k] + pre] = make_uint2(up | neg, szx[k]);
                     }
                     if (pi) {
-                        const int32_t C = one_comp ? 0 : __ldg(P.comp + x[k]);
+                        const int32_t C = one_comp ? 0 : __ldg(P.comp_i + x[k]);
                         if (C == P.cbig) atomicAdd(&s_big[bk[k]], 1u);
                         else atomicAdd(P.s1 + (size_t)bk[k] * P.ncomp + C, 1u);
                     }
@@ -694,12 +702,13 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
             const uint32_t x = __ldcg(P.qv + qi);
             uint32_t pre, up, neg, pi, p = 0, szx;
             if (L == 0) {
-                const int32_t C = one_comp ? 0 : __ldg(P.comp + x);
+                const int32_t C = one_comp ? 0 : __ldg(P.comp_i + x);
                 pre = (uint32_t)__ldg(P.coff + C);
                 up = pre;
                 neg = 0;
                 pi = 0;
-                szx = 1 + (kDescent ? (uint32_t)__ldcg(P.sz64 + nb + x) : __ldcg(P.size + nb + x));
+                szx = 1 + (kDescent ? (uint32_t)__ldcg(P.sz64 + nb + x)
+                                    : __ldcg(P.size + (size_t)b * P.szn + szi(P, x)));
             } else {
                 const uint32_t pq = __ldcg(P.parq + qi);
                 p = pq & kIdMask;
@@ -726,7 +735,7 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
                 if (L > 0) P.clist[__ldcg(P.cstart + nb + p) + __ldcg(P.cidxq + qi)] = pre;
             }
             if (pi) {
-                const int32_t C = one_comp ? 0 : __ldg(P.comp + x);
+                const int32_t C = one_comp ? 0 : __ldg(P.comp_i + x);
                 if (C == P.cbig) atomicAdd(&s_big[b], 1u);
                 else atomicAdd(P.s1 + (size_t)b * P.ncomp + C, 1u);
             }
@@ -769,24 +778,36 @@ __global__ void k_child_counts(TreeParams P, int64_t cnt) {
         P.cstart[i] = (uint32_t)(P.sz64[i] >> 32);
 }
 
-// caller trees (push BFS): parent keys -> parent | neg << 31 in queue order
-__global__ void k_pkey_to_parq(const unsigned long long *pkeyq, uint32_t *parq, int64_t cnt) {
+// caller trees (push BFS): parent keys -> parent | neg << 31 in queue order,
+// and the level lists translated to internal ids (the labelling passes' and
+// the walk's index space); level-0 entries (roots) point at themselves
+__global__ void k_pkey_to_parq(TreeParams P, const unsigned long long *pkeyq) {
+    const int64_t cnt = (int64_t)P.vbase[P.depth[0] + 1];
+    const int64_t nroots = (int64_t)P.vbase[1];
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < cnt;
          i += (int64_t)gridDim.x * blockDim.x) {
-        const unsigned long long k = pkeyq[i];
-        parq[i] = ((uint32_t)(k >> 1) & kIdMask) | ((uint32_t)k << 31);
+        const uint32_t vi = P.brank[P.qv[i]];
+        P.qv[i] = vi;
+        if (i < nroots) {
+            P.parq[i] = vi;
+        } else {
+            const unsigned long long k = pkeyq[i];
+            P.parq[i] = P.brank[(uint32_t)(k >> 1) & kIdMask] | ((uint32_t)k << 31);
+        }
     }
 }
 
 // ---------------------------------------------------------------------------
 // debug views of one tree (b = 0): parent / dist / size by vertex
 // ---------------------------------------------------------------------------
-__global__ void k_debug_tree(TreeParams P, int32_t *parent, int32_t *dist, int32_t *size) {
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < P.n;
-         v += (int64_t)gridDim.x * blockDim.x) {
+__global__ void k_debug_tree(TreeParams P, int32_t *parent, int32_t *dist, int32_t *size, int32_t *pre) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t v = P.bord[i];   // labels live in internal ids; outputs by original id
         parent[v] = -1;
         dist[v] = 0;
-        size[v] = 1 + (P.sz64 ? (int32_t)(uint32_t)P.sz64[v] : (int32_t)P.size[v]);
+        size[v] = 1 + (P.sz64 ? (int32_t)(uint32_t)P.sz64[i] : (int32_t)P.size[szi(P, (uint32_t)i)]);
+        pre[v] = (int32_t)(P.pp[i] & kIdMask);
     }
 }
 
@@ -799,9 +820,9 @@ __global__ void k_debug_tree_scatter(TreeParams P, int64_t nqueued, int32_t *par
             const int mid = (lo + hi) >> 1;
             if ((int64_t)P.vbase[mid] <= i) lo = mid; else hi = mid;
         }
-        const uint32_t v = P.qv[i];
+        const uint32_t v = P.bord[P.qv[i]];
         dist[v] = lo;
-        parent[v] = lo == 0 ? -1 : (int32_t)(P.parq[i] & kIdMask);
+        parent[v] = lo == 0 ? -1 : (int32_t)P.bord[P.parq[i] & kIdMask];
     }
 }
 
@@ -830,12 +851,15 @@ static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_
                               bool descent, int b0 = 0) {
     TreeParams P;
     P.row_ptr = g.row_ptr; P.adj = g.adj;
-    P.comp = g.comp; P.coff = g.coff; P.cverts = g.cverts;
+    P.brank = g.brank; P.bord = g.bord;
+    P.comp = g.comp; P.comp_i = g.comp_i; P.coff = g.coff; P.cverts = g.cverts;
     P.n = g.n; P.ncomp = g.ncomp; P.nw = (g.n + 3) / 4; P.cbig = g.cbig;
     P.B = B; P.ls = g.n + 2;
     P.vst = ws.vst; P.qv = ws.qv; P.qs = ws.qs; P.qr = ws.qr; P.pkeyq = ws.pkeyq;
     P.lvl = ws.lvl; P.vbase = ws.vbase;
     P.size = descent ? nullptr : ws.size;
+    P.szn = size_slots(g.n);
+    P.szmask = (uint32_t)(P.szn - 1);
     P.sz64 = descent ? ws.sz64 : nullptr;
     P.parq = ws.parq; P.offq = ws.offq; P.szq = ws.szq;
     P.cidxq = descent ? ws.cidxq : nullptr;
@@ -850,7 +874,7 @@ static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_
     if (b0) {
         const size_t nb = (size_t)b0 * g.n, lb = (size_t)b0 * P.ls;
         P.qv += nb; P.parq += nb; P.offq += nb; P.szq += nb; P.pp += nb; P.rec += nb;
-        if (P.size) P.size += nb;
+        if (P.size) P.size += (size_t)b0 * P.szn;
         if (P.sz64) P.sz64 += nb;
         if (P.cidxq) P.cidxq += nb;
         if (P.cstart) P.cstart += nb;
@@ -879,7 +903,7 @@ static int set_window(cudaStream_t st, void *base, size_t bytes, size_t persist)
 
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
                    cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub,
-                   int recpass, size_t persist, int sampler) {
+                   int recpass, size_t persist, int sampler, const BfsOpts &bfs) {
     if (descent) recpass = 0;
     // co-resident grid sizes, recomputed when the device changes
     static int bfs_blocks = 0, up_blocks[2] = {0, 0}, down_blocks[2] = {0, 0}, blocks_dev = -1;
@@ -896,7 +920,7 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
     if (ev) GB_CUDA_TRY(cudaEventRecord(ev[0], st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.s1, 0, sizeof(uint32_t) * (size_t)B * g.ncomp, st));
     if (descent) GB_CUDA_TRY(cudaMemsetAsync(ws.sz64, 0, sizeof(unsigned long long) * (size_t)B * g.n, st));
-    else GB_CUDA_TRY(cudaMemsetAsync(ws.size, 0, sizeof(uint32_t) * (size_t)B * g.n, st));
+    else GB_CUDA_TRY(cudaMemsetAsync(ws.size, 0, sizeof(uint32_t) * (size_t)B * size_slots(g.n), st));
     k_batch_prep<<<1, kMaxBatch, 0, st>>>(P);
     ++*launches;
     // f.3: a uniform random spanning tree (B = 1), then the caller-tree path
@@ -920,7 +944,7 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
         int rc = launch_coop((const void *)k_bfs, bfs_blocks, P, st);
         if (rc) return rc;
         ++*launches;
-        k_pkey_to_parq<<<(unsigned)std::min<int64_t>((g.n + 255) / 256, 4096), 256, 0, st>>>(ws.pkeyq, ws.parq, g.n);
+        k_pkey_to_parq<<<(unsigned)std::min<int64_t>((g.n + 255) / 256, 4096), 256, 0, st>>>(P, ws.pkeyq);
         ++*launches;
     } else {
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[1], st));
@@ -928,7 +952,8 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
         o.qv = ws.qv; o.parq = ws.parq; o.pp = ws.pp; o.rec = ws.rec;
         o.crec = descent ? ws.crec : nullptr;
         o.lvl = ws.lvl; o.vbase = ws.vbase; o.depth = ws.depth; o.maxd = ws.maxd; o.tkey = ws.tkey;
-        int rc = run_msbfs(g, ws, B, o, st, launches);
+        int rc = bfs.kind == 1 ? run_msbfs(g, ws, B, o, st, launches)
+                               : run_tbfs(g, ws, B, o, st, launches, bfs.group, bfs.push_k);
         if (rc) return rc;
     }
     GB_CUDA_TRY(cudaGetLastError());
@@ -972,7 +997,7 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
 }
 
 int debug_tree_views(const Graph &g, Workspace &ws, bool descent, int32_t *d_parent,
-                     int32_t *d_dist, int32_t *d_size, cudaStream_t st) {
+                     int32_t *d_dist, int32_t *d_size, int32_t *d_pre, cudaStream_t st) {
     TreeParams P = make_params(g, ws, 1, nullptr, descent);
     int32_t depth = 0;
     GB_CUDA_TRY(cudaMemcpyAsync(&depth, ws.depth, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
@@ -980,7 +1005,7 @@ int debug_tree_views(const Graph &g, Workspace &ws, bool descent, int32_t *d_par
     uint32_t nq = 0;
     GB_CUDA_TRY(cudaMemcpyAsync(&nq, ws.vbase + depth + 1, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
     GB_CUDA_TRY(cudaStreamSynchronize(st));
-    k_debug_tree<<<256, 256, 0, st>>>(P, d_parent, d_dist, d_size);
+    k_debug_tree<<<256, 256, 0, st>>>(P, d_parent, d_dist, d_size, d_pre);
     k_debug_tree_scatter<<<256, 256, 0, st>>>(P, nq, d_parent, d_dist);
     GB_CUDA_TRY(cudaGetLastError());
     GB_CUDA_TRY(cudaStreamSynchronize(st));

@@ -145,11 +145,17 @@ def set_option(key: str, value: int):
     _check(lib().gb_set_option(key.encode(), int(value)))
 
 
-def balance_host(num_trees, seed):
-    """gb_balance with host outputs: (edge_flip_counts uint32[m], vertex_agree uint32[n])."""
+def balance_host(num_trees, seed, out=None):
+    """gb_balance with host outputs: (edge_flip_counts uint32[m], vertex_agree uint32[n]).
+    `out` = optional caller arrays (uint32, >= max(m,1) and n long; e.g. pinned)."""
     n, m, _ = graph_info()
-    cnt = np.zeros(max(m, 1), np.uint32)
-    agree = np.zeros(n, np.uint32)
+    if out is not None:
+        cnt, agree = out
+        if cnt.dtype != np.uint32 or agree.dtype != np.uint32 or len(cnt) < max(m, 1) or len(agree) < n:
+            raise GraphBError(GB_EINVAL, "out arrays must be uint32 of length >= m and n")
+    else:
+        cnt = np.zeros(max(m, 1), np.uint32)
+        agree = np.zeros(n, np.uint32)
     _check(lib().gb_balance(int(num_trees), int(seed) & (2**64 - 1), _ptr(cnt), _ptr(agree)))
     return cnt[:m], agree
 
@@ -161,6 +167,8 @@ def balance_range(t_begin, t_end, t_stride, seed, d_edge_cnt, d_vertex_agree, st
         if not (t.is_cuda and t.dtype == torch.int32 and t.is_contiguous()):
             raise GraphBError(GB_EINVAL, "outputs must be contiguous int32 CUDA tensors")
     s = stream.cuda_stream if stream is not None else torch.cuda.current_stream().cuda_stream
+    if s == 0:
+        s = 1   # torch's legacy default stream: cudaStreamLegacy (NULL would mean the library's own stream)
     _check(lib().gb_balance_range(int(t_begin), int(t_end), int(t_stride), int(seed) & (2**64 - 1),
                                   ctypes.c_void_p(d_edge_cnt.data_ptr()),
                                   ctypes.c_void_p(d_vertex_agree.data_ptr()), ctypes.c_void_p(s)))
@@ -244,11 +252,11 @@ def balance_given_tree(parent):
 
 
 def stats():
-    ints = np.zeros(9, np.int64)
+    ints = np.zeros(11, np.int64)
     ph = np.zeros(len(PHASES), np.float64)
-    lib().gb_get_stats(_ptr(ints), 9, _ptr(ph), len(PHASES))
+    lib().gb_get_stats(_ptr(ints), 11, _ptr(ph), len(PHASES))
     keys = ("trees", "sum_cycle_len", "cycles", "launches", "batches", "max_depth", "batch",
-            "cycle_group", "harary_violations")
+            "cycle_group", "harary_violations", "sub", "bfs_group")
     d = {k: int(v) for k, v in zip(keys, ints)}
     d["phase_ms"] = {k: float(v) for k, v in zip(PHASES, ph)}
     return d
