@@ -87,6 +87,7 @@ struct State {
     Graph g;
     Workspace ws;
     bool ws_descent = false;
+    bool ws_irec = false;
     cudaStream_t stream = nullptr;
     int32_t *d_cnt = nullptr, *d_agree = nullptr;  // gb_balance's device counters
     int32_t *d_given = nullptr;                    // caller tree (gb_balance_given_tree)
@@ -106,7 +107,7 @@ constexpr int64_t kStateSlots = 2 * kRecCap;  // open-addressing table of gb_clo
 
 static void free_ws(Workspace &w) {
     void *ptrs[] = {w.vst, w.qv, w.qs, w.qr, w.pkeyq, w.lvl, w.vbase, w.size, w.sz64,
-                    w.parq, w.offq, w.szq, w.pp, w.rec, w.fbits, w.s1, w.tkey, w.depth,
+                    w.parq, w.offq, w.szq, w.pp, w.rec, w.irec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
                     w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof,
                     w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey, w.tbm, w.tbhbest, w.tbhpos, w.tbhlev};
@@ -126,9 +127,14 @@ static BfsOpts bfs_opts() {
     return b;
 }
 
+// record layout: 0 = records by internal id (walk 0, one level per record),
+// 1 = pp + pre-indexed records (walk 1, option jump)
+static bool irec_layout() { return S.opt.walk == 0 && S.opt.jump == 1; }
+
 static size_t per_tree_bytes(const Graph &g, bool descent) {
     const size_t n = (size_t)g.n;
-    size_t b = 44 * n + 32 + 4 * (size_t)((g.m + 31) / 32) + 4 * (size_t)g.ncomp;
+    size_t b = 36 * n + 32 + 4 * (size_t)((g.m + 31) / 32) + 4 * (size_t)g.ncomp;
+    b += irec_layout() ? 16 * n : 12 * n;
     if (descent) b += 24 * n;
     return b;
 }
@@ -144,7 +150,8 @@ static size_t per_tree_bytes(const Graph &g, bool descent) {
     } while (0)
 
 static int ensure_workspace(int B, bool descent) {
-    if (S.ws.B >= B && descent == S.ws_descent) return GB_OK;
+    const bool irec = irec_layout();
+    if (S.ws.B >= B && descent == S.ws_descent && irec == S.ws_irec) return GB_OK;
     B = std::max(B, S.ws.B);
     free_ws(S.ws);
     Workspace &w = S.ws;
@@ -185,8 +192,13 @@ static int ensure_workspace(int B, bool descent) {
     ALLOC(w.parq, Bn);
     ALLOC(w.offq, Bn);
     ALLOC(w.szq, Bn);
-    ALLOC(w.pp, Bn);
-    ALLOC(w.rec, Bn);
+    if (irec) {
+        ALLOC(w.irec, Bn);
+    } else {
+        ALLOC(w.pp, Bn);
+        ALLOC(w.rec, Bn);
+    }
+    w.irec_layout = irec;
     ALLOC(w.fbits, (int64_t)B * words);
     ALLOC(w.s1, (int64_t)B * g.ncomp);
     ALLOC(w.tkey, kMaxBatch);
@@ -208,6 +220,7 @@ static int ensure_workspace(int B, bool descent) {
     w.B = B;
     w.n = n;
     S.ws_descent = descent;
+    S.ws_irec = irec;
     return GB_OK;
 }
 

@@ -33,7 +33,8 @@ struct CycleParams {
     const uint2 *edges;    // [m] {u, v | neg<<31} by eid, internal ids (the labels' index space)
     int64_t n, m;
     const uint32_t *pp;    // [B][n] pre | pi<<31
-    const uint2 *rec;      // [B][n] pre-indexed {up | neg<<31, size}
+    const uint2 *rec;      // [B][n] pre-indexed {up | neg<<31, size}                (layout 1)
+    const uint4 *irec;     // [B][n] by internal id {parent | neg, pre | pi, size, 0} (layout 0)
     const uint2 *crec;     // [B][n] pre-indexed {child-list start, #children}
     const uint32_t *clist; // children pre IDs, per parent ascending
     uint32_t *fbits;       // [B][words]
@@ -137,6 +138,63 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_two_ended(CycleParams P)
             const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
             if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
             // per-tree cycle statistics and state signature
+            warp_stats(lane, g, k, cyc, flip != 0, e, s_k, s_c, s_sig);
+        }
+    }
+    __syncthreads();
+    flush_stats(P, s_k, s_c, s_sig);
+}
+
+// Layout 0 (default): the same two-ended walk over records indexed by
+// internal vertex id, {parent | neg<<31, pre | pi<<31, size}.  The endpoints'
+// records are the first two loads (no separate label lookup), the tree-edge
+// test is on the parent words, and a climb step is one 16-byte gather; the
+// ancestors the climbs share (hubs and other high-degree vertices, internal
+// ids at the front) sit in a dense, L2-hot region.
+__global__ void __launch_bounds__(kCycleBlock) k_cycles_irec(CycleParams P) {
+    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup], s_sig[kMaxGroup];
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; s_sig[i] = 0; }
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t word = gw; word < P.words; word += nw) {
+        const int64_t e = word * 32 + lane;
+        const bool valid = e < P.m;
+        uint2 ed = valid ? __ldg(P.edges + e) : make_uint2(0, 0);
+        const uint32_t u = ed.x, v = ed.y & kIdMask, nege = ed.y >> 31;
+        for (int g = 0; g < P.G; g++) {
+            const uint4 *rec = P.irec + (size_t)(P.b0 + g) * P.n;
+            uint32_t flip = 0, k = 0;
+            bool cyc = false;
+            if (valid) {
+                uint4 rx = __ldg(rec + u), ry = __ldg(rec + v);
+                // tree edge iff one endpoint is the other's parent (simple graph)
+                if ((rx.x & kIdMask) != v && (ry.x & kIdMask) != u) {
+                    cyc = true;
+                    const uint32_t px = rx.y & kIdMask, py = ry.y & kIdMask;
+                    uint32_t c = 0;
+                    k = 1;
+                    bool ax = is_anc(px, rx.z, py), ay = is_anc(py, ry.z, px);
+                    while (!(ax && ay)) {
+                        if (!ax) {
+                            c ^= rx.x;
+                            rx = __ldg(rec + (rx.x & kIdMask));
+                            k++;
+                            ax = is_anc(rx.y & kIdMask, rx.z, py);
+                        }
+                        if (!ay) {
+                            c ^= ry.x;
+                            ry = __ldg(rec + (ry.x & kIdMask));
+                            k++;
+                            ay = is_anc(ry.y & kIdMask, ry.z, px);
+                        }
+                    }
+                    flip = (c >> 31) ^ nege;
+                }
+            }
+            const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
+            if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
             warp_stats(lane, g, k, cyc, flip != 0, e, s_k, s_c, s_sig);
         }
     }
@@ -350,7 +408,7 @@ __global__ void k_accumulate_edges(const uint32_t *__restrict__ fbits, int64_t w
 }
 
 // (labels in internal ids i; the counter of the original vertex bord[i])
-__global__ void k_accumulate_agree(const uint32_t *__restrict__ pp, const uint32_t *__restrict__ s1,
+__global__ void k_accumulate_agree(const uint32_t *__restrict__ pp, int ps, const uint32_t *__restrict__ s1,
                                    const int32_t *__restrict__ comp_i, const int32_t *__restrict__ coff,
                                    const uint32_t *__restrict__ bord,
                                    int64_t n, int64_t ncomp, int B, int32_t *__restrict__ agree) {
@@ -361,7 +419,7 @@ __global__ void k_accumulate_agree(const uint32_t *__restrict__ pp, const uint32
         int32_t d = 0;
         for (int b = 0; b < B; b++) {
             const uint32_t ones = __ldg(s1 + (size_t)b * ncomp + C);
-            const uint32_t mine = (__ldg(pp + (size_t)b * n + v) >> 31) ? ones : cs - ones;
+            const uint32_t mine = (__ldg(pp + ((size_t)b * n + v) * ps) >> 31) ? ones : cs - ones;
             const uint32_t other = cs - mine;
             d += mine > other ? 2 : (mine == other ? 1 : 0);
         }
@@ -382,6 +440,9 @@ int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool desce
     P.jrec = ws.jrec;
     P.edges = g.edges_i; P.n = g.n; P.m = g.m;
     P.pp = ws.pp; P.rec = ws.rec; P.crec = ws.crec; P.clist = ws.clist;
+    P.irec = ws.irec;
+    const bool irec = ws.irec_layout && !descent;
+    if (irec) jump = 1;
     P.fbits = ws.fbits; P.tstat = ws.tstat;
     P.words = (g.m + 31) / 32;
     if (P.words == 0) return GB_OK;
@@ -396,7 +457,8 @@ int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool desce
             else k_build_jump<4><<<dim3(bx, P.G), 256, 0, st>>>(ws.rec + (size_t)b0 * g.n, ws.jrec, g.n);
             ++*launches;
         }
-        if (descent) k_cycles_descent<<<grid, kCycleBlock, 0, st>>>(P);
+        if (irec) k_cycles_irec<<<grid, kCycleBlock, 0, st>>>(P);
+        else if (descent) k_cycles_descent<<<grid, kCycleBlock, 0, st>>>(P);
         else if (jump == 2) k_cycles_jump<2><<<grid, kCycleBlock, 0, st>>>(P);
         else if (jump == 4) k_cycles_jump<4><<<grid, kCycleBlock, 0, st>>>(P);
         else k_cycles_two_ended<<<grid, kCycleBlock, 0, st>>>(P);
@@ -414,7 +476,7 @@ int run_batch_accumulate(const Graph &g, Workspace &ws, int B, int32_t *d_cnt, i
         ++*launches;
     }
     k_accumulate_agree<<<grid_cap(g.n, 256, g.num_sms, 16), 256, 0, st>>>(
-        ws.pp, ws.s1, g.comp_i, g.coff, g.bord, g.n, g.ncomp, B, d_agree);
+        label_words(ws), label_stride(ws), ws.s1, g.comp_i, g.coff, g.bord, g.n, g.ncomp, B, d_agree);
     ++*launches;
     GB_CUDA_TRY(cudaGetLastError());
     return GB_OK;

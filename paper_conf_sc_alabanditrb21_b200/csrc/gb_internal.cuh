@@ -158,8 +158,13 @@ struct Workspace {
     uint32_t *parq = nullptr;  // q: parent id | neg(parent edge)<<31
     uint32_t *offq = nullptr;  // q: offset of the child's range inside its parent's
     uint32_t *szq = nullptr;   // q: subtree size
-    uint32_t *pp = nullptr;    // v: pre | pi<<31  (pi = root-path parity)
-    uint2 *rec = nullptr;      // pre: {up pre | neg<<31, size}
+    uint32_t *pp = nullptr;    // v: pre | pi<<31  (pi = root-path parity)      [layout 1]
+    uint2 *rec = nullptr;      // pre: {up pre | neg<<31, size}                  [layout 1]
+    uint4 *irec = nullptr;     // v: {parent | neg<<31, pre | pi<<31, size, 0}   [layout 0]
+    bool irec_layout = false;  // layout 0 (walk 0 with one level per record, the default):
+                               // records indexed by internal vertex id, written by the
+                               // top-down pass itself; layout 1 (walk 1, option jump):
+                               // pp by vertex + records by pre order (k_rec_scatter)
     uint32_t *fbits = nullptr; // [B][ceil(m/32)] flip bitmask
     void *wbuf = nullptr;      // option "sampler" = 1, "wilson" = 1: cycle-popping state (20n bytes)
     void *wseq = nullptr;      // option "sampler" = 1, 2: [W] trees of per-thread sampler state (13n bytes each);
@@ -276,6 +281,7 @@ int run_dfs_batch(const Graph &g, Workspace &ws, int W, cudaStream_t st, int64_t
 struct MsBfsOut {
     uint32_t *qv, *parq, *pp;
     uint2 *rec, *crec;
+    uint4 *irec;
     uint64_t *lvl;
     uint32_t *vbase;
     int32_t *depth, *maxd;
@@ -295,6 +301,13 @@ int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool desce
 
 int run_batch_accumulate(const Graph &g, Workspace &ws, int B, int32_t *d_cnt,
                          int32_t *d_agree, cudaStream_t st, int64_t *launches);
+
+// the word holding pre | pi<<31 of vertex v in tree b: pp (layout 1) or the
+// second word of the internal-id record (layout 0)
+inline uint32_t *label_words(Workspace &ws) {
+    return ws.irec_layout ? reinterpret_cast<uint32_t *>(ws.irec) + 1 : ws.pp;
+}
+inline int label_stride(const Workspace &ws) { return ws.irec_layout ? 4 : 1; }
 
 // f.2: Harary sides of the B trees of a batch by the L224 procedure (replaces
 // the pi bits of pp and the per-component counts s1); d_bad counts edges

@@ -59,6 +59,7 @@ struct MsParams {
     const uint64_t *tkey;
     uint32_t *qv, *parq, *pp;
     uint2 *rec, *crec;
+    uint4 *irec;
     uint64_t *lvl;
     uint32_t *vbase;
     int32_t *depth, *maxd;
@@ -442,9 +443,13 @@ __global__ void k_ms_roots(MsParams P) {
         if (P.brow[ri + 1] == P.brow[ri]) {
             // isolated vertex: a one-vertex tree, finished here (pi = 0)
             const uint32_t pre = (uint32_t)P.coff[C];
-            P.pp[nb + ri] = pre;
-            P.rec[nb + pre] = make_uint2(pre, 1u);
-            if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
+            if (P.irec) {
+                P.irec[nb + ri] = make_uint4(ri, pre, 1u, 0u);
+            } else {
+                P.pp[nb + ri] = pre;
+                P.rec[nb + pre] = make_uint2(pre, 1u);
+                if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
+            }
             continue;
         }
         const unsigned long long old = atomicAdd((unsigned long long *)(P.lvl + b * P.ls), 1ull << 32);
@@ -829,7 +834,7 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
     P.fcnt = reinterpret_cast<uint32_t *>(ws.msflag + 4);
     P.push_div = 32;   // measured on C3: 32 and 128 equal (bfs 59.0 ms / 100 trees), 8 worse (61.3)
     P.flag = ws.msflag; P.mscnt = ws.mscnt;
-    P.tkey = o.tkey; P.qv = o.qv; P.parq = o.parq; P.pp = o.pp; P.rec = o.rec; P.crec = o.crec;
+    P.tkey = o.tkey; P.qv = o.qv; P.parq = o.parq; P.pp = o.pp; P.rec = o.rec; P.crec = o.crec; P.irec = o.irec;
     P.lvl = o.lvl; P.vbase = o.vbase; P.depth = o.depth; P.maxd = o.maxd;
     P.prof = ws.msprof;
     GB_CUDA_TRY(cudaMemsetAsync(ws.vis, 0, sizeof(unsigned long long) * (size_t)g.n, st));

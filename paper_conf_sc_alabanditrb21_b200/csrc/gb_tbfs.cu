@@ -56,6 +56,7 @@ struct TbParams {
     const uint64_t *tkey;         // [G]
     uint32_t *qv, *parq, *pp;     // tree stride n
     uint2 *rec, *crec;
+    uint4 *irec;
     uint64_t *lvl;                // [G][ls]: vertex count << 32 | degree sum, per level
     uint32_t *vbase;              // [G][ls]
     int32_t *depth, *maxd;
@@ -119,9 +120,13 @@ __global__ void k_tb_roots(TbParams P) {
         if (deg == 0) {
             // isolated vertex: a one-vertex tree, finished here (pi = 0)
             const uint32_t pre = (uint32_t)P.coff[C];
-            P.pp[nb + ri] = pre;
-            P.rec[nb + pre] = make_uint2(pre, 1u);
-            if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
+            if (P.irec) {
+                P.irec[nb + ri] = make_uint4(ri, pre, 1u, 0u);
+            } else {
+                P.pp[nb + ri] = pre;
+                P.rec[nb + pre] = make_uint2(pre, 1u);
+                if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
+            }
             continue;
         }
         const unsigned long long old = atomicAdd((unsigned long long *)(P.lvl + g * P.ls), (1ull << 32) | deg);
@@ -462,6 +467,7 @@ int run_tbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStream
         P.tkey = o.tkey + b0;
         P.qv = o.qv + nb; P.parq = o.parq + nb; P.pp = o.pp + nb; P.rec = o.rec + nb;
         P.crec = o.crec ? o.crec + nb : nullptr;
+        P.irec = o.irec ? o.irec + nb : nullptr;
         P.lvl = o.lvl + lb; P.vbase = o.vbase + lb;
         P.depth = o.depth + b0; P.maxd = o.maxd;
         P.push_k = push_k;

@@ -52,6 +52,7 @@ struct TreeParams {
     uint32_t *parq, *offq, *szq, *cidxq;
     uint32_t *pp;
     uint2 *rec;
+    uint4 *irec;                 // layout 0: {parent | neg, pre | pi, size, 0} by internal id
     uint32_t *s1;
     const uint64_t *tkey;
     int32_t *depth, *maxd;
@@ -121,9 +122,14 @@ __device__ __forceinline__ void place_root(const TreeParams &P, int b, int64_t C
     const uint32_t pre = (uint32_t)P.coff[C];
     if (deg == 0) {
         // isolated vertex: a one-vertex tree, finished here (pi = 0)
-        P.pp[nb + P.brank[r]] = pre;
-        P.rec[nb + pre] = make_uint2(pre, 1u);
-        if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
+        const uint32_t ri = P.brank[r];
+        if (P.irec) {
+            P.irec[nb + ri] = make_uint4(ri, pre, 1u, 0u);
+        } else {
+            P.pp[nb + ri] = pre;
+            P.rec[nb + pre] = make_uint2(pre, 1u);
+            if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
+        }
         if (P.visited) atomicAdd(P.visited + b, 1ull);
         return;
     }
@@ -668,18 +674,24 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
                 }
 #pragma unroll
                 for (int k = 0; k < kILP; k++)
-                    if (bk[k] >= 0) ppp[k] = __ldcg(P.pp + nbk[k] + (pq[k] & kIdMask));
+                    if (bk[k] >= 0)
+                        ppp[k] = P.irec ? __ldcg(reinterpret_cast<const uint32_t *>(P.irec + nbk[k] + (pq[k] & kIdMask)) + 1)
+                                        : __ldcg(P.pp + nbk[k] + (pq[k] & kIdMask));
 #pragma unroll
                 for (int k = 0; k < kILP; k++) {
                     if (bk[k] < 0) continue;
                     const uint32_t up = ppp[k] & kIdMask, neg = pq[k] & kNegBit;
                     const uint32_t pre = up + off[k];
                     const uint32_t pi = (ppp[k] & kNegBit) ^ neg;
-                    P.pp[nbk[k] + x[k]] = pre | pi;
-                    if (P.recpass) {
+                    if (P.irec) {
+                        // layout 0: the record by internal id, complete here
+                        P.irec[nbk[k] + x[k]] = make_uint4(pq[k], pre | pi, szx[k], 0u);
+                    } else if (P.recpass) {
+                        P.pp[nbk[k] + x[k]] = pre | pi;
                         GB_QST(P.parq + qi[k], up | neg);
                         GB_QST(P.offq + qi[k], pre);
                     } else {
+                        P.pp[nbk[k] + x[k]] = pre | pi;
                         P.rec[nbk[k] + pre] = make_uint2(up | neg, szx[k]);
                     }
                     if (pi) {
@@ -712,19 +724,23 @@ __global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
             } else {
                 const uint32_t pq = __ldcg(P.parq + qi);
                 p = pq & kIdMask;
-                const uint32_t ppp = __ldcg(P.pp + nb + p);
+                const uint32_t ppp = P.irec ? __ldcg(reinterpret_cast<const uint32_t *>(P.irec + nb + p) + 1)
+                                            : __ldcg(P.pp + nb + p);
                 up = ppp & kIdMask;
                 pre = up + __ldcg(P.offq + qi);
                 neg = pq & kNegBit;
                 pi = (ppp & kNegBit) ^ neg;
                 szx = __ldcg(P.szq + qi);
             }
-            P.pp[nb + x] = pre | pi;
-            if (!kDescent && P.recpass) {
+            if (!kDescent && P.irec) {
+                P.irec[nb + x] = make_uint4(L == 0 ? x : (p | neg), pre | pi, szx, 0u);
+            } else if (!kDescent && P.recpass) {
+                P.pp[nb + x] = pre | pi;
                 P.parq[qi] = up | neg;
                 P.offq[qi] = pre;
                 P.szq[qi] = szx;
             } else {
+                P.pp[nb + x] = pre | pi;
                 P.rec[nb + pre] = make_uint2(up | neg, szx);
             }
             if (kDescent) {
@@ -807,7 +823,7 @@ __global__ void k_debug_tree(TreeParams P, int32_t *parent, int32_t *dist, int32
         parent[v] = -1;
         dist[v] = 0;
         size[v] = 1 + (P.sz64 ? (int32_t)(uint32_t)P.sz64[i] : (int32_t)P.size[szi(P, (uint32_t)i)]);
-        pre[v] = (int32_t)(P.pp[i] & kIdMask);
+        pre[v] = (int32_t)((P.irec ? P.irec[i].y : P.pp[i]) & kIdMask);
     }
 }
 
@@ -864,6 +880,7 @@ static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_
     P.parq = ws.parq; P.offq = ws.offq; P.szq = ws.szq;
     P.cidxq = descent ? ws.cidxq : nullptr;
     P.pp = ws.pp; P.rec = ws.rec; P.s1 = ws.s1; P.tkey = ws.tkey; P.depth = ws.depth;
+    P.irec = (ws.irec_layout && !descent) ? ws.irec : nullptr;
     P.maxd = ws.maxd; P.given = given;
     P.cstart = descent ? ws.cstart : nullptr;
     P.clist = descent ? ws.clist : nullptr;
@@ -873,7 +890,10 @@ static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_
     P.prof = ws.msprof ? ws.msprof + 1024 : nullptr;
     if (b0) {
         const size_t nb = (size_t)b0 * g.n, lb = (size_t)b0 * P.ls;
-        P.qv += nb; P.parq += nb; P.offq += nb; P.szq += nb; P.pp += nb; P.rec += nb;
+        P.qv += nb; P.parq += nb; P.offq += nb; P.szq += nb;
+        if (P.pp) P.pp += nb;
+        if (P.rec) P.rec += nb;
+        if (P.irec) P.irec += nb;
         if (P.size) P.size += (size_t)b0 * P.szn;
         if (P.sz64) P.sz64 += nb;
         if (P.cidxq) P.cidxq += nb;
@@ -904,7 +924,7 @@ static int set_window(cudaStream_t st, void *base, size_t bytes, size_t persist)
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
                    cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub,
                    int recpass, size_t persist, int sampler, const BfsOpts &bfs) {
-    if (descent) recpass = 0;
+    if (descent || ws.irec_layout) recpass = 0;
     // co-resident grid sizes, recomputed when the device changes
     static int bfs_blocks = 0, up_blocks[2] = {0, 0}, down_blocks[2] = {0, 0}, blocks_dev = -1;
     if (blocks_dev != g.dev) {
@@ -950,6 +970,7 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[1], st));
         MsBfsOut o;
         o.qv = ws.qv; o.parq = ws.parq; o.pp = ws.pp; o.rec = ws.rec;
+        o.irec = (ws.irec_layout && !descent) ? ws.irec : nullptr;
         o.crec = descent ? ws.crec : nullptr;
         o.lvl = ws.lvl; o.vbase = ws.vbase; o.depth = ws.depth; o.maxd = ws.maxd; o.tkey = ws.tkey;
         int rc = bfs.kind == 1 ? run_msbfs(g, ws, B, o, st, launches)

@@ -405,6 +405,36 @@ def test_c3_amazon_sampled_trees():
     assert np.array_equal(d["flip"], og.balance_tree(parent)[0])
 
 
+@pytest.mark.slow
+def test_c3_amazon_cloud_subset_bit_exact():
+    """C3 (10M / 22M) at full size: a strided subset of the bench step's 100
+    trees (3, 27, 51, 75, 99) through gb_balance_range into device counters;
+    every edge flip count and every vertex agree count equals the oracle's
+    (Alg. 1 L96-L108 on the same trees, the L224 Harary procedure)."""
+    import torch
+    g, T, _ = graphgen.config("c3")
+    graphb.load_graph(g)
+    cnt = torch.zeros(g.m, dtype=torch.int32, device="cuda")
+    agr = torch.zeros(g.n, dtype=torch.int32, device="cuda")
+    graphb.balance_range(3, T, 24, 1, cnt, agr)
+    torch.cuda.synchronize()
+    st = graphb.stats()
+    assert st["trees"] == 5
+    oc, oa, ost = oracle.Graph.from_csr(g).balance(T, 1, t_begin=3, stride=24, with_stats=True)
+    assert np.array_equal(cnt.cpu().numpy().astype(np.uint32), oc)
+    assert np.array_equal(agr.cpu().numpy().astype(np.uint32), oa)
+    ids, per = graphb.tree_stats()
+    assert list(ids) == [3, 27, 51, 75, 99]
+    assert np.array_equal(per, ost)        # sum k, cycles, depth, state signature
+
+
+def test_rmat20_full_cloud_bit_exact():
+    """Graph500 R-MAT scale 20 (the C5 recipe at 1/64 of the size): the whole
+    frustration cloud of 8 trees, every counter, against the oracle."""
+    g = graphgen.rmat(20, 16, 0.5, 3, name="rmat20")
+    check_cloud(g, 8, 2)
+
+
 @pytest.mark.parametrize("which", ["er", "forest", "c2"])
 def test_ingest_edge_ids_and_components(which):
     """§8 a.1: edge table by eid (rank of (min,max)), eid of every slot, and
