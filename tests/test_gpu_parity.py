@@ -6,6 +6,8 @@ size, flips).  Pre-order IDs are not unique (the sibling order is free,
 reading R5), so they are checked for validity instead."""
 from __future__ import annotations
 
+import os
+
 import numpy as np
 import pytest
 
@@ -91,17 +93,29 @@ def test_c1_config_exact():
     assert st["trees"] == 1
 
 
-@pytest.mark.parametrize("walk", [0, 1])
+@pytest.mark.parametrize("walk", [0, 1, 2])
 def test_tree_stages_match_oracle(walk):
     g = graphgen.er(3000, 12000, 0.3, 4)
     check_tree_debug(g, 5, range(6), walk=walk)
 
 
-@pytest.mark.parametrize("walk", [0, 1])
-def test_power_law_hubs_multi_batch(walk):
-    """Hubs (Chung-Lu) + several batches + cycle groups smaller than a batch."""
+@pytest.mark.parametrize("walk,linear", [(0, 0), (1, 0), (1, 1), (2, 0)])
+def test_power_law_hubs_multi_batch(walk, linear):
+    """Hubs (Chung-Lu, children lists of thousands) + several batches + cycle
+    groups smaller than a batch; walk 1 with 32-ary pivots and with linear
+    int4 ballot rounds, walk 2 = the paper's partitioned two-word edge lists
+    (L238-L244)."""
     g = graphgen.chung_lu(20000, 90000, 2500, 0.75, 0.25, 3)
-    check_cloud(g, 37, 11, batch=16, cycle_group=5, walk=walk)
+    check_cloud(g, 37, 11, batch=16, cycle_group=5, walk=walk, desc_linear=linear)
+
+
+@pytest.mark.parametrize("walk", [1, 2])
+def test_paper_walks_on_forests_and_degenerate_trees(walk):
+    """Walks 1 and 2 on a forest with isolated vertices (roots without a
+    parent edge) and on a star (one hub with every vertex as a child)."""
+    check_cloud(graphgen.er(5000, 3000, 0.4, 2), 9, 3, walk=walk)
+    check_cloud(graphgen.star(300), 4, 1, walk=walk)
+    check_cloud(graphgen.complete(40, lambda u, v: -1 if (u * v) % 3 == 1 else 1), 6, 2, walk=walk, desc_linear=1)
 
 
 @pytest.mark.parametrize("jump,recpass,sub", [(1, 0, 0), (1, 1, 1), (2, 1, 0), (2, 0, 3), (4, 1, 1), (4, 0, 0)])
@@ -502,6 +516,20 @@ def _climb_checks(g, d, sample_edges, rng):
     return int((~tree).sum()), k
 
 
+def _c5_golden():
+    rows = {"trees": []}
+    with open(os.path.join(os.path.dirname(__file__), "golden", "c5_rmat26_trees.txt")) as f:
+        for line in f:
+            w = line.split()
+            if not w or w[0].startswith("#"):
+                continue
+            if w[0] == "graph":
+                rows["graph"] = (int(w[1]), int(w[2]), w[3], w[4])
+            elif w[0] == "tree":
+                rows["trees"].append((int(w[1]), int(w[2]), int(w[3]), int(w[4]), int(w[5], 16), w[6], w[7]))
+    return rows
+
+
 @pytest.mark.slow
 def test_c5_rmat26_capacity_and_sampled_cycles():
     """C5 (RMAT scale 26, ~1 B generated edges) on one B200: loads, balances
@@ -531,3 +559,24 @@ def test_c5_rmat26_capacity_and_sampled_cycles():
         assert d["parent"][w] == best
     nonc, _ = _climb_checks(g, d, rng.integers(0, len(g.col), 20000), rng)
     assert nonc > 1000
+    # whole trees bit-exact against the oracle: tests/golden/c5_rmat26_trees.txt
+    # holds the oracle's one-tree counters (sha256) and statistics, written by
+    # tools/make_c5_golden.py (graphgen + oracle/ only); its graph line pins
+    # the generated input
+    import hashlib
+    import torch
+    gold = _c5_golden()
+    sha = lambda a: hashlib.sha256(np.ascontiguousarray(a).tobytes()).hexdigest()
+    assert gold["graph"] == (g.n, g.m, sha(g.col.astype("<i4")), sha(g.sign.astype("i1")))
+    assert len(gold["trees"]) >= 2
+    cnt_d = torch.zeros(m, dtype=torch.int32, device="cuda")
+    agr_d = torch.zeros(n, dtype=torch.int32, device="cuda")
+    for t, sk, nc, dep, sig, hc, ha in gold["trees"]:
+        cnt_d.zero_()
+        agr_d.zero_()
+        graphb.balance_range(t, t + 1, 1, 1, cnt_d, agr_d)
+        torch.cuda.synchronize()
+        _, per1 = graphb.tree_stats()
+        assert tuple(int(x) for x in per1[0]) == (sk, nc, dep, sig)
+        assert sha(cnt_d.cpu().numpy().astype("<u4")) == hc
+        assert sha(agr_d.cpu().numpy().astype("<u4")) == ha
