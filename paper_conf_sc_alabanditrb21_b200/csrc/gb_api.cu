@@ -48,7 +48,8 @@ void arena_free_all() {
 struct Options {
     int64_t batch = 0;       // 0 = auto
     int64_t cycle_group = 0; // 0 = auto
-    int64_t walk = 0;        // 0 two-ended, 1 Alg. 3 descent
+    int64_t walk = 0;        // 0 two-ended, 1 Alg. 3 descent (child lists), 2 the paper's edge lists (L238-L244)
+    int64_t desc_linear = 0; // walk 1: 1 = linear int4 ballot rounds over the child starts, 0 = 32-ary pivots
     int64_t timing = 0;
     int64_t sub = 0;         // trees per labelling launch (0 = auto)
     int64_t msprof = 0;      // record BFS phase timestamps (gb_msbfs_profile)
@@ -110,7 +111,8 @@ static void free_ws(Workspace &w) {
                     w.parq, w.offq, w.szq, w.pp, w.rec, w.irec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
                     w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof,
-                    w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey, w.tbm, w.tbhbest, w.tbhpos, w.tbhlev};
+                    w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey, w.tbm, w.tbhbest, w.tbhpos, w.tbhlev,
+                    w.ptbase, w.ptnbr, w.ptrng};
     for (void *p : ptrs) if (p) cudaFree(p);
     w = Workspace();
 }
@@ -210,12 +212,12 @@ static int ensure_workspace(int B, bool descent) {
         ALLOC(w.sz64, Bn);
         ALLOC(w.cidxq, Bn);
         ALLOC(w.cstart, Bn);
-        ALLOC(w.clist, Bn);
+        ALLOC(w.clist, Bn + 4);   // + 4: the 16-byte loads of walk 1's linear scan
         ALLOC(w.crec, Bn);
         w.scan_tmp_elems = scan_tmp_elems(Bn);
         ALLOC(w.scan_tmp, (int64_t)w.scan_tmp_elems);
     } else {
-        ALLOC(w.size, (int64_t)B * size_slots(n));
+        ALLOC(w.size, Bn);
     }
     w.B = B;
     w.n = n;
@@ -288,18 +290,20 @@ static int auto_batch(int64_t ntrees) {
     // the multi-source BFS holds one bit per tree in a 64-bit word
     if (S.opt.batch > 0) return (int)std::min<int64_t>(S.opt.batch, kMsBatch);
     const size_t have = S.free_at_load;
-    int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk == 1));
+    int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk >= 1));
     int64_t b = std::min<int64_t>({ntrees, (int64_t)kMsBatch, std::max<int64_t>(bm, 1)});
     return (int)std::max<int64_t>(b, 1);
 }
 
-// trees per labelling launch: large graphs label one tree at a time so its
-// random-access array (40 MB for a 10M-vertex tree) stays L2-resident
-// (measured on C3: 1 tree 38.9 ms / 100 trees top-down, 2 trees 49.5, 4 trees
-// 58.4); small graphs label the whole batch
+// trees per labelling launch: small graphs label the whole batch in one
+// launch; large ones a few trees at a time, so the random-access working set
+// (size counters + records, 20 B per vertex and tree) stays mostly in L2 while
+// the per-level grid barriers are shared (measured on C3 with internal ids,
+// bottom-up + top-down per 100 trees: 1 tree 55.8 ms, 2 trees 52.4, 4 trees
+// 50.8; with round 1's random original ids 1 tree was best)
 static int auto_sub(int B) {
     if (S.opt.sub > 0) return (int)std::min<int64_t>(S.opt.sub, B);
-    if (S.g.n >= (1 << 22)) return 1;
+    if (S.g.n >= (1 << 22)) return std::min(B, 4);
     return B;
 }
 
@@ -364,7 +368,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     T.pending = true;
     const int64_t K = t_end > t_begin ? (t_end - t_begin + stride - 1) / stride : 0;
     if (K == 0) return GB_OK;
-    const bool descent = S.opt.walk == 1;
+    const bool descent = S.opt.walk >= 1;   // walks 1 and 2 need the child lists
     int B = auto_batch(K);
     // walk 1 keeps child lists of a whole batch in one 32-bit index space
     if (descent) B = (int)std::min<int64_t>(B, std::max<int64_t>(1, ((1ll << 32) - 1) / S.g.n));
@@ -445,7 +449,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
                             bfs_opts());
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
-        rc = run_batch_cycles(S.g, S.ws, nb, G, descent, st, &T.launches, jump);
+        rc = run_batch_cycles(S.g, S.ws, nb, G, (int)S.opt.walk, st, &T.launches, jump, (int)S.opt.desc_linear);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[5], st));
         if (S.opt.harary) {
@@ -479,7 +483,7 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
     Stats &T = S.st;
     drop_events(T);
     T = Stats();
-    int rc = ensure_workspace(1, S.opt.walk == 1);
+    int rc = ensure_workspace(1, S.opt.walk >= 1);
     if (rc) return rc;
     cudaStream_t st = S.stream;
     k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, 1, seed, t, 1);
@@ -497,7 +501,7 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
         if (rc) return rc;
         d_given = reinterpret_cast<const int32_t *>(S.ws.wseq);
     }
-    rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk == 1, 1,
+    rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk >= 1, 1,
                         0, 0, d_given ? 0 : (int)S.opt.sampler, bfs_opts());
     if (rc) return rc;
     if (user_tree) {
@@ -510,7 +514,7 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
             return GB_EINVAL;
         }
     }
-    rc = run_batch_cycles(S.g, S.ws, 1, 1, S.opt.walk == 1, st, &T.launches);
+    rc = run_batch_cycles(S.g, S.ws, 1, 1, (int)S.opt.walk, st, &T.launches, 1, (int)S.opt.desc_linear);
     if (rc) return rc;
     GB_CUDA_TRY(cudaStreamSynchronize(st));
     return GB_OK;
@@ -656,7 +660,11 @@ int gb_set_option(const char *key, int64_t value) {
     if (!key) { set_error("NULL option"); return GB_EINVAL; }
     if (!strcmp(key, "batch")) { if (value < 0) return GB_EINVAL; S.opt.batch = value; }
     else if (!strcmp(key, "cycle_group")) { if (value < 0) return GB_EINVAL; S.opt.cycle_group = value; }
-    else if (!strcmp(key, "walk")) { if (value != 0 && value != 1) return GB_EINVAL; S.opt.walk = value; }
+    else if (!strcmp(key, "walk")) {
+        if (value < 0 || value > 2) { set_error("walk must be 0 (two-ended), 1 (Alg. 3 descent) or 2 (paper edge lists)"); return GB_EINVAL; }
+        S.opt.walk = value;
+    }
+    else if (!strcmp(key, "desc_linear")) S.opt.desc_linear = value != 0;
     else if (!strcmp(key, "timing")) S.opt.timing = value != 0;
     else if (!strcmp(key, "sub")) { if (value < 0) return GB_EINVAL; S.opt.sub = value; }
     else if (!strcmp(key, "msprof")) S.opt.msprof = value != 0;
@@ -742,7 +750,7 @@ int gb_tree_debug(int64_t t, uint64_t seed, int32_t *parent, int32_t *dist, int3
     const int64_t n = S.g.n;
     int32_t *d_tmp = nullptr;
     GB_CUDA_TRY(cudaMalloc(&d_tmp, sizeof(int32_t) * 4 * n));
-    rc = debug_tree_views(S.g, S.ws, S.opt.walk == 1, d_tmp, d_tmp + n, d_tmp + 2 * n, d_tmp + 3 * n, S.stream);
+    rc = debug_tree_views(S.g, S.ws, S.opt.walk >= 1, d_tmp, d_tmp + n, d_tmp + 2 * n, d_tmp + 3 * n, S.stream);
     if (rc) { cudaFree(d_tmp); return rc; }
     std::vector<int32_t> h(4 * n);
     cudaError_t ce = cudaMemcpy(h.data(), d_tmp, sizeof(int32_t) * 4 * n, cudaMemcpyDeviceToHost);

@@ -41,6 +41,10 @@ struct CycleParams {
     unsigned long long *tstat;  // [B][3] {sum cycle length, cycles, state signature}
     int64_t words;
     int b0, G;             // trees b0 .. b0+G-1 of the batch
+    int linear;            // walk 1: child search by linear int4 ballot rounds (1) or 32-ary pivots (0)
+    const uint32_t *tbase; // walk 2: [n+1] start of each vertex's tree-edge list (pre order)
+    const uint32_t *tnbr;  // walk 2: [2n] neighbour (pre id) of each tree-edge record
+    const uint2 *trng;     // walk 2: [2n] {begin | inverted<<31, end | neg<<31} (L238)
     uint2 *jrec;           // [G][n][K] K-level ancestor records (walk 0, option "jump" = K > 1)
 };
 
@@ -360,6 +364,38 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_descent(CycleParams P) {
                     // the last child start <= ty (its range holds ty)
                     const uint2 cr = __ldg(crec + cx);
                     uint32_t lo = cr.x, cnt = cr.y;
+                    if (P.linear) {
+                        // linear ballot rounds over the sorted child starts,
+                        // four per lane with one 16-byte load (128 per round):
+                        // the round that holds the first start > ty decides
+                        const uint32_t a0 = lo & ~3u, end = lo + cnt;
+                        for (uint32_t base = a0;; base += 128) {
+                            const uint32_t q = base + 4 * lane;
+                            uint4 v4 = make_uint4(~0u, ~0u, ~0u, ~0u);
+                            if (q < end) v4 = __ldg(reinterpret_cast<const uint4 *>(P.clist + q));
+                            // positions outside [lo, end) never count
+                            const bool b0 = q >= lo && q < end && v4.x <= ty;
+                            const bool b1 = q + 1 >= lo && q + 1 < end && v4.y <= ty;
+                            const bool b2 = q + 2 >= lo && q + 2 < end && v4.z <= ty;
+                            const bool b3 = q + 3 >= lo && q + 3 < end && v4.w <= ty;
+                            const uint32_t m0 = __ballot_sync(0xFFFFFFFFu, b0), m1 = __ballot_sync(0xFFFFFFFFu, b1);
+                            const uint32_t m2 = __ballot_sync(0xFFFFFFFFu, b2), m3 = __ballot_sync(0xFFFFFFFFu, b3);
+                            const uint32_t tot = __popc(m0) + __popc(m1) + __popc(m2) + __popc(m3);
+                            const uint32_t avail = min(end, base + 128) - max(lo, base);
+                            if (tot < avail || base + 128 >= end) {
+                                // sorted: the starts <= ty are a prefix; the child is the last of them
+                                const uint32_t before = max(lo, base) - lo;
+                                lo = lo + before + tot - 1;
+                                cnt = 1;
+                                break;
+                            }
+                        }
+                        const uint32_t ch = __ldg(P.clist + lo);
+                        cpar ^= __ldg(rec + ch).x;   // neg bit of the edge into ch
+                        cx = ch;
+                        steps++;
+                        continue;
+                    }
                     while (cnt > 32) {
                         const uint32_t step = (cnt + 31) >> 5;
                         const uint32_t pos = lane * step;
@@ -384,6 +420,110 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_descent(CycleParams P) {
             if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
             warp_stats(lane, g, k, cyc, flip != 0, e, s_k, s_c, s_sig);
         }
+    }
+    __syncthreads();
+    flush_stats(P, s_k, s_c, s_sig);
+}
+
+// ---------------------------------------------------------------------------
+// walk 2 (§8 f.1): the paper's own traversal data structure (§3.2.1-3.2.2,
+// L238-L244).  Per tree, in pre-order ID space, every vertex x has a
+// partitioned tree-edge list with the parent edge first, then the child edges
+// (ascending); each edge is two words (L238): begin | inverted << 31 and
+// end | sign << 31, next to the neighbour id.  The parent edge's range is x's
+// own subtree range, inverted (L212: it leads to every ID outside it).  The
+// walk is Alg. 3 as written (L190-L201): from v_src, scan the list for the
+// edge whose (possibly inverted) range holds v_dst, count its sign, move,
+// until v_dst -- one thread per non-tree edge, as the paper's lane per
+// non-tree edge (L307), reading record pairs with 16-byte loads.
+// ---------------------------------------------------------------------------
+__global__ void k_paper_counts(const uint2 *__restrict__ crec, int64_t n, uint32_t *__restrict__ tcnt) {
+    for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x <= n;
+         x += (int64_t)gridDim.x * blockDim.x)
+        tcnt[x] = x < n ? 1u + __ldg(&crec[x].y) : 0u;   // parent slot + children
+}
+
+// thread per pre ID x: the parent-edge record of x's own list, and the record
+// of edge parent(x) -> x in the parent's list (its position = x's rank among
+// the sorted children, found by binary search)
+__global__ void k_paper_fill(const uint2 *__restrict__ rec, const uint2 *__restrict__ crec,
+                             const uint32_t *__restrict__ clist, const uint32_t *__restrict__ tbase,
+                             int64_t n, uint32_t *__restrict__ tnbr, uint2 *__restrict__ trng) {
+    for (int64_t xi = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; xi < n;
+         xi += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t x = (uint32_t)xi;
+        const uint2 r = __ldg(rec + x);
+        const uint32_t up = r.x & kIdMask, neg = r.x & kNegBit, end = x + r.y - 1;
+        const uint32_t s = __ldg(tbase + x);
+        if (up == x) {   // a root: no parent edge; an empty range that never matches
+            tnbr[s] = x;
+            trng[s] = make_uint2(1u, 0u);
+            continue;
+        }
+        tnbr[s] = up;
+        trng[s] = make_uint2(x | kNegBit, end | neg);          // inverted: everything outside x's subtree
+        const uint2 cp = __ldg(crec + up);
+        uint32_t lo = 0, hi = cp.y;                              // clist[cp.x + lo] <= x < clist[cp.x + hi]
+        while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (__ldg(clist + cp.x + mid) <= x) lo = mid; else hi = mid;
+        }
+        const uint32_t sp = __ldg(tbase + up) + 1 + lo;
+        tnbr[sp] = x;
+        trng[sp] = make_uint2(x, end | neg);
+    }
+}
+
+__device__ __forceinline__ bool paper_hit(uint2 w, uint32_t y) {
+    const uint32_t b = w.x & kIdMask, e = w.y & kIdMask;
+    const bool in = (y - b) <= (e - b) && b <= e;
+    return in != (bool)(w.x >> 31);
+}
+
+__global__ void __launch_bounds__(kCycleBlock) k_cycles_paper(CycleParams P) {
+    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup], s_sig[kMaxGroup];
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; s_sig[i] = 0; }
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const size_t nb = (size_t)P.b0 * P.n;
+    const uint2 *rec = P.rec + nb;
+    for (int64_t word = gw; word < P.words; word += nw) {
+        const int64_t e = word * 32 + lane;
+        const bool valid = e < P.m;
+        uint2 ed = valid ? __ldg(P.edges + e) : make_uint2(0, 0);
+        const uint32_t u = ed.x, v = ed.y & kIdMask, nege = ed.y >> 31;
+        uint32_t flip = 0, k = 0;
+        bool cyc = false;
+        if (valid) {
+            uint32_t x = __ldg(P.pp + nb + u) & kIdMask;
+            const uint32_t y = __ldg(P.pp + nb + v) & kIdMask;
+            // tree edge iff one endpoint is the other's parent (simple graph)
+            if ((__ldg(rec + x).x & kIdMask) != y && (__ldg(rec + y).x & kIdMask) != x) {
+                cyc = true;
+                uint32_t c = 0;
+                k = 1;
+                while (x != y) {
+                    const uint32_t s0 = __ldg(P.tbase + x), s1 = __ldg(P.tbase + x + 1);
+                    uint32_t s = s0 & ~1u;
+                    bool found = false;
+                    for (; s < s1; s += 2) {
+                        const uint4 two = __ldg(reinterpret_cast<const uint4 *>(P.trng + s));
+                        if (s >= s0 && paper_hit(make_uint2(two.x, two.y), y)) { found = true; break; }
+                        if (s + 1 < s1 && paper_hit(make_uint2(two.z, two.w), y)) { s++; found = true; break; }
+                    }
+                    if (!found) { k = 0; break; }   // cannot happen on a valid tree; no endless loop
+                    c ^= __ldg(P.trng + s).y;                 // the sign bit of the traversed edge
+                    x = __ldg(P.tnbr + s);
+                    k++;
+                }
+                flip = (c >> 31) ^ nege;
+            }
+        }
+        const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
+        if (lane == 0) P.fbits[(size_t)P.b0 * P.words + word] = bits;
+        warp_stats(lane, 0, k, cyc, flip != 0, e, s_k, s_c, s_sig);
     }
     __syncthreads();
     flush_stats(P, s_k, s_c, s_sig);
@@ -433,20 +573,29 @@ static unsigned grid_cap(int64_t work, int threads, int sms, int per_sm) {
     return (unsigned)std::max<int64_t>(1, std::min(b, cap));
 }
 
-int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool descent,
-                     cudaStream_t st, int64_t *launches, int jump) {
+int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, int walk,
+                     cudaStream_t st, int64_t *launches, int jump, int linear) {
     CycleParams P;
-    if (descent || !ws.jrec) jump = 1;
+    const bool descent = walk == 1, paper = walk == 2;
+    if (walk != 0 || !ws.jrec) jump = 1;
     P.jrec = ws.jrec;
     P.edges = g.edges_i; P.n = g.n; P.m = g.m;
     P.pp = ws.pp; P.rec = ws.rec; P.crec = ws.crec; P.clist = ws.clist;
     P.irec = ws.irec;
-    const bool irec = ws.irec_layout && !descent;
+    P.linear = linear;
+    P.tbase = nullptr; P.tnbr = nullptr; P.trng = nullptr;
+    const bool irec = ws.irec_layout && walk == 0;
     if (irec) jump = 1;
     P.fbits = ws.fbits; P.tstat = ws.tstat;
     P.words = (g.m + 31) / 32;
     if (P.words == 0) return GB_OK;
+    if (paper) group = 1;   // one tree's lists at a time
     group = std::max(1, std::min(group, kMaxGroup));
+    if (paper && !ws.ptbase) {
+        GB_CUDA_TRY(cudaMalloc(&ws.ptbase, sizeof(uint32_t) * (size_t)(2 * (g.n + 1))));
+        GB_CUDA_TRY(cudaMalloc(&ws.ptnbr, sizeof(uint32_t) * (size_t)(2 * g.n + 2)));
+        GB_CUDA_TRY(cudaMalloc(&ws.ptrng, sizeof(uint2) * (size_t)(2 * g.n + 2)));
+    }
     for (int b0 = 0; b0 < B; b0 += group) {
         P.b0 = b0;
         P.G = std::min(group, B - b0);
@@ -457,7 +606,20 @@ int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool desce
             else k_build_jump<4><<<dim3(bx, P.G), 256, 0, st>>>(ws.rec + (size_t)b0 * g.n, ws.jrec, g.n);
             ++*launches;
         }
-        if (irec) k_cycles_irec<<<grid, kCycleBlock, 0, st>>>(P);
+        if (paper) {
+            // the paper's partitioned tree-edge lists of tree b0 (pre order)
+            const size_t nb = (size_t)b0 * g.n;
+            uint32_t *tcnt = ws.ptbase + (g.n + 1);
+            const unsigned gx = grid_cap(g.n + 1, 256, g.num_sms, 8);
+            k_paper_counts<<<gx, 256, 0, st>>>(ws.crec + nb, g.n, tcnt);
+            int rc = exclusive_scan_u32(tcnt, ws.ptbase, g.n + 1, ws.scan_tmp, ws.scan_tmp_elems, st, launches);
+            if (rc) return rc;
+            k_paper_fill<<<gx, 256, 0, st>>>(ws.rec + nb, ws.crec + nb, ws.clist, ws.ptbase, g.n, ws.ptnbr, ws.ptrng);
+            *launches += 2;
+            P.tbase = ws.ptbase; P.tnbr = ws.ptnbr; P.trng = ws.ptrng;
+            k_cycles_paper<<<grid, kCycleBlock, 0, st>>>(P);
+        }
+        else if (irec) k_cycles_irec<<<grid, kCycleBlock, 0, st>>>(P);
         else if (descent) k_cycles_descent<<<grid, kCycleBlock, 0, st>>>(P);
         else if (jump == 2) k_cycles_jump<2><<<grid, kCycleBlock, 0, st>>>(P);
         else if (jump == 4) k_cycles_jump<4><<<grid, kCycleBlock, 0, st>>>(P);

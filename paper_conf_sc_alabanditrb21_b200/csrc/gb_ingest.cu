@@ -13,7 +13,6 @@
 #include "gb_internal.cuh"
 #include "../../include/graphb.h"
 
-#include <cub/device/device_radix_sort.cuh>
 
 #include <algorithm>
 #include <vector>
@@ -119,6 +118,97 @@ int exclusive_scan_u32(const uint32_t *in, uint32_t *out, int64_t count, uint32_
     k_scan_partials<<<1, 1024, 0, st>>>(tmp, nb);
     k_scan_down<<<(unsigned)nb, kScanThreads, 0, st>>>(in, out, count, tmp);
     *launches += 3;
+    GB_CUDA_TRY(cudaGetLastError());
+    return GB_OK;
+}
+
+// ---------------------------------------------------------------------------
+// Stable LSD radix sort of (key, value) pairs, 8-bit digits (used twice at
+// ingest: vertices grouped by component, and the degree-sorted view).  One
+// warp owns a tile of 256 consecutive elements: pass 1 counts the tile's
+// digits, an exclusive scan over the digit-major count matrix gives every
+// (digit, tile) its output run, pass 2 walks the tile in order, 32 elements
+// at a time, ranking equal digits with __match_any_sync -- stable.
+// ---------------------------------------------------------------------------
+constexpr int kRsWarps = 8;
+constexpr int kRsTile = 256;      // elements per warp tile
+
+__device__ __forceinline__ uint32_t rs_digit(uint32_t k, int shift, uint32_t flip) {
+    return ((k >> shift) & 255u) ^ flip;
+}
+
+__global__ void k_rs_hist(const uint32_t *__restrict__ keys, int64_t n, int shift, uint32_t flip,
+                          uint32_t *__restrict__ hist, int64_t ntiles) {
+    __shared__ uint32_t h[kRsWarps][256];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    for (int d = lane; d < 256; d += 32) h[wid][d] = 0;
+    __syncwarp();
+    const int64_t tile = (int64_t)blockIdx.x * kRsWarps + wid;
+    if (tile >= ntiles) return;
+    const int64_t base = tile * kRsTile;
+    for (int c = 0; c < kRsTile / 32; c++) {
+        const int64_t i = base + c * 32 + lane;
+        if (i < n) atomicAdd(&h[wid][rs_digit(__ldg(keys + i), shift, flip)], 1u);
+    }
+    __syncwarp();
+    for (int d = lane; d < 256; d += 32) hist[(int64_t)d * ntiles + tile] = h[wid][d];
+}
+
+__global__ void k_rs_scatter(const uint32_t *__restrict__ kin, const uint32_t *__restrict__ vin,
+                             uint32_t *__restrict__ kout, uint32_t *__restrict__ vout, int64_t n,
+                             int shift, uint32_t flip, const uint32_t *__restrict__ off, int64_t ntiles) {
+    __shared__ uint32_t run[kRsWarps][256];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int64_t tile = (int64_t)blockIdx.x * kRsWarps + wid;
+    if (tile >= ntiles) return;      // warp-uniform
+    for (int d = lane; d < 256; d += 32) run[wid][d] = __ldg(off + (int64_t)d * ntiles + tile);
+    __syncwarp();
+    const uint32_t lt = (1u << lane) - 1u;
+    const int64_t base = tile * kRsTile;
+    for (int c = 0; c < kRsTile / 32; c++) {
+        const int64_t i = base + c * 32 + lane;
+        const bool valid = i < n;
+        const uint32_t k = valid ? __ldg(kin + i) : 0u;
+        const uint32_t d = rs_digit(k, shift, flip);
+        const uint32_t peers = __match_any_sync(0xFFFFFFFFu, valid ? d : 0x100u + (uint32_t)lane);
+        const uint32_t b = valid ? run[wid][d] : 0u;
+        __syncwarp();
+        if (valid) {
+            const uint32_t pos = b + __popc(peers & lt);
+            kout[pos] = k;
+            vout[pos] = __ldg(vin + i);
+            if (lane == __ffs(peers) - 1) run[wid][d] = b + __popc(peers);
+        }
+        __syncwarp();
+    }
+}
+
+// temporaries: 2n (ping-pong keys / values) + 256 * ceil(n / 256) (counts)
+size_t radix_tmp_elems(int64_t n) { return (size_t)(2 * n + 256 * ((n + kRsTile - 1) / kRsTile) + 64); }
+
+// keys_in -> keys_out, vals_in -> vals_out over key bits [0, bits), stable;
+// descending order of keys if `desc` (equal keys keep their input order)
+static int radix_sort_pairs(const uint32_t *kin, uint32_t *kout, const uint32_t *vin, uint32_t *vout,
+                            int64_t n, int bits, bool desc, uint32_t *tmp, uint32_t *scan_tmp,
+                            size_t scan_elems, cudaStream_t st, int64_t *launches) {
+    if (n <= 0) return GB_OK;
+    const int64_t ntiles = (n + kRsTile - 1) / kRsTile;
+    uint32_t *ktmp = tmp, *vtmp = tmp + n, *hist = tmp + 2 * n;
+    const int passes = std::max(1, (bits + 7) / 8);
+    const uint32_t flip = desc ? 255u : 0u;
+    const unsigned blocks = (unsigned)((ntiles + kRsWarps - 1) / kRsWarps);
+    const uint32_t *ks = kin, *vs = vin;
+    for (int p = 0; p < passes; p++) {
+        const bool to_out = ((passes - 1 - p) % 2) == 0;
+        uint32_t *kd = to_out ? kout : ktmp, *vd = to_out ? vout : vtmp;
+        k_rs_hist<<<blocks, kRsWarps * 32, 0, st>>>(ks, n, 8 * p, flip, hist, ntiles);
+        int rc = exclusive_scan_u32(hist, hist, 256 * ntiles, scan_tmp, scan_elems, st, launches);
+        if (rc) return rc;
+        k_rs_scatter<<<blocks, kRsWarps * 32, 0, st>>>(ks, vs, kd, vd, n, 8 * p, flip, hist, ntiles);
+        *launches += 2;
+        ks = kd;
+        vs = vd;
+    }
     GB_CUDA_TRY(cudaGetLastError());
     return GB_OK;
 }
@@ -495,14 +585,16 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
         ++*launches;
         int bits = 1;
         while (bits < 32 && (1ll << bits) < nc) bits++;
-        size_t sort_bytes = 0;
-        ING_TRY(cub::DeviceRadixSort::SortPairs(nullptr, sort_bytes, keys, skeys, ids, (uint32_t *)g.cverts,
-                                                (int)n, 0, bits, st));
-        char *sort_tmp = nullptr;
-        ING_ALLOC(sort_tmp, kArSortTmp, sort_bytes);
-        ING_TRY(cub::DeviceRadixSort::SortPairs(sort_tmp, sort_bytes, keys, skeys, ids, (uint32_t *)g.cverts,
-                                                (int)n, 0, bits, st));
-        *launches += 4;
+        uint32_t *sort_tmp = nullptr;
+        ING_ALLOC(sort_tmp, kArSortTmp, radix_tmp_elems(n));
+        {
+            const size_t rs_scan = scan_tmp_elems(256 * ((n + 255) / 256));
+            uint32_t *rs_stmp = nullptr;
+            ING_ALLOC(rs_stmp, kArRsScan, rs_scan);
+            rc = radix_sort_pairs(keys, skeys, ids, (uint32_t *)g.cverts, n, bits, false, sort_tmp,
+                                  rs_stmp, rs_scan, st, launches);
+            if (rc) goto done;
+        }
         k_comp_offsets<<<grid_for(n, 256, sms), 256, 0, st>>>(skeys, n, nc, g.coff);
         ++*launches;
         ING_TRY(cudaMemsetAsync(big, 0, sizeof(unsigned long long), st));
@@ -530,14 +622,18 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
         ING_ALLOC(g.borig, kArBorig, slots);
         k_degrees<<<grid_for(n, 256, sms), 256, 0, st>>>(g.row_ptr, n, deg, ids);
         ++*launches;
-        size_t sort_bytes = 0;
-        ING_TRY(cub::DeviceRadixSort::SortPairsDescending(nullptr, sort_bytes, deg, sdeg, ids, g.bord,
-                                                          (int)n, 0, 32, st));
-        char *sort_tmp = nullptr;
-        ING_ALLOC(sort_tmp, kArSortTmp, sort_bytes);
-        ING_TRY(cub::DeviceRadixSort::SortPairsDescending(sort_tmp, sort_bytes, deg, sdeg, ids, g.bord,
-                                                          (int)n, 0, 32, st));
-        *launches += 4;
+        {
+            // degrees are < n (simple graph): ceil(log2 n) key bits
+            int dbits = 1;
+            while (dbits < 32 && (1ll << dbits) < n) dbits++;
+            uint32_t *sort_tmp = nullptr;
+            ING_ALLOC(sort_tmp, kArSortTmp, radix_tmp_elems(n));
+            const size_t rs_scan = scan_tmp_elems(256 * ((n + 255) / 256));
+            uint32_t *rs_stmp = nullptr;
+            ING_ALLOC(rs_stmp, kArRsScan, rs_scan);
+            rc = radix_sort_pairs(deg, sdeg, ids, g.bord, n, dbits, true, sort_tmp, rs_stmp, rs_scan, st, launches);
+            if (rc) goto done;
+        }
         ING_TRY(cudaMemsetAsync(cnt2, 0, 2 * sizeof(unsigned long long), st));
         k_view_rank<<<grid_for(n, 256, sms), 256, 0, st>>>(g.bord, sdeg, n, g.brank, cnt2);
         ++*launches;

@@ -203,6 +203,10 @@ struct Workspace {
     uint32_t *cstart = nullptr;// v: start of the child list (global position)
     uint32_t *clist = nullptr; // [B*n] children pre IDs, grouped by parent, ascending
     uint2 *crec = nullptr;     // pre: {cstart, #children}
+    // walk 2 (the paper's lists, one tree at a time)
+    uint32_t *ptbase = nullptr;  // [n+1] list starts (pre order) + [n+1] counts
+    uint32_t *ptnbr = nullptr;   // [2n] neighbour pre IDs
+    uint2 *ptrng = nullptr;      // [2n] two-word range/sign records
     uint32_t *scan_tmp = nullptr;
     size_t scan_tmp_elems = 0;
 };
@@ -244,7 +248,7 @@ enum ArenaSlot {
     kArRowPtr64, kArCol, kArSign, kArErr, kArRowPtr, kArAdj, kArAdjEid, kArEdges, kArComp,
     kArCverts, kArUptr, kArUpc, kArEbase, kArScanTmp, kArLab, kArFlag, kArRank, kArCoff,
     kArBrow, kArBadj, kArBorig, kArBord, kArBrank, kArItems, kArDeg, kArSortTmp, kArCkeys,
-    kArEdgesI, kArCompI, kArSlots
+    kArEdgesI, kArCompI, kArRsScan, kArSlots
 };
 void *arena(int slot, size_t bytes);   // nullptr on allocation failure (error set)
 void arena_free_all();
@@ -296,8 +300,10 @@ int run_tbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStream
 int debug_tree_views(const Graph &g, Workspace &ws, bool descent, int32_t *d_parent,
                      int32_t *d_dist, int32_t *d_size, int32_t *d_pre, cudaStream_t st);
 
-int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, bool descent,
-                     cudaStream_t st, int64_t *launches, int jump = 1);
+// walk: 0 two-ended, 1 Alg. 3 descent over child lists, 2 the paper's
+// partitioned two-word edge lists (linear scan)
+int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, int walk,
+                     cudaStream_t st, int64_t *launches, int jump = 1, int linear = 0);
 
 int run_batch_accumulate(const Graph &g, Workspace &ws, int B, int32_t *d_cnt,
                          int32_t *d_agree, cudaStream_t st, int64_t *launches);

@@ -61,21 +61,24 @@ struct TreeParams {
     uint2 *crec;                 // walk 1
     unsigned long long *visited; // [B] vertices reached (given-tree validation)
     unsigned long long *prof;    // option "msprof": [256][4] level timestamps (gb_label_profile)
-    uint32_t szmask;             // szn - 1
-    int64_t szn;                 // size counters per tree (power of two >= n)
+    uint32_t szmask;             // (power of two >= n) - 1
+    int64_t szn;                 // size counters per tree (n)
     int recpass;                 // walk 0: top-down leaves {up | neg, size} and pre in queue
                                  // order; k_rec_scatter writes rec[pre] afterwards
 };
 
 // Slot of vertex i's subtree-size counter: a multiplicative scramble of the
-// id, i * 0x9E3779B1 mod szn (odd multiplier: a bijection on [0, szn)).
-// Internal ids put the hubs -- the parents of most vertices -- next to each
-// other, and the atomics of the bottom-up pass then queue on a few hot L2
-// sectors; scrambled, a hot counter's sector mates are unrelated (mostly
-// cold) vertices.  (Bit reversal does the same but turns consecutive ids into
-// power-of-two strides: measured slower.)
+// id, y = i * 0x9E3779B1 mod 2^k (2^k >= n; an odd multiplier permutes
+// [0, 2^k)), repeated while y >= n (cycle walking: a permutation of [0, n),
+// under 2 steps on average).  Internal ids put the hubs -- the parents of
+// most vertices -- next to each other, and the atomics of the bottom-up pass
+// then queue on a few hot L2 sectors; scrambled, a hot counter's sector mates
+// are unrelated (mostly cold) vertices (C3: bottom-up 42 -> 30 ms per 100
+// trees; bit reversal over 2^k slots measured the same).
 __device__ __forceinline__ uint32_t szi(const TreeParams &P, uint32_t i) {
-    return (i * 0x9E3779B1u) & P.szmask;
+    uint32_t y = (i * 0x9E3779B1u) & P.szmask;
+    while (y >= (uint32_t)P.n) y = (y * 0x9E3779B1u) & P.szmask;
+    return y;
 }
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
@@ -621,7 +624,7 @@ __global__ void __launch_bounds__(kBlock) k_bottom_up(TreeParams P) {
 // rec[pre] = {pre(parent) | neg<<31, size} used by the cycle walk.
 // ---------------------------------------------------------------------------
 template <bool kDescent>
-__global__ void __launch_bounds__(kBlock) k_top_down(TreeParams P) {
+__global__ void __launch_bounds__(kBlock, 4) k_top_down(TreeParams P) {
     cg::grid_group grid = cg::this_grid();
     __shared__ LevelTable T;
     __shared__ int32_t s_depth[kMaxBatch];
@@ -874,8 +877,8 @@ static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_
     P.vst = ws.vst; P.qv = ws.qv; P.qs = ws.qs; P.qr = ws.qr; P.pkeyq = ws.pkeyq;
     P.lvl = ws.lvl; P.vbase = ws.vbase;
     P.size = descent ? nullptr : ws.size;
-    P.szn = size_slots(g.n);
-    P.szmask = (uint32_t)(P.szn - 1);
+    P.szn = g.n;
+    P.szmask = (uint32_t)(size_slots(g.n) - 1);
     P.sz64 = descent ? ws.sz64 : nullptr;
     P.parq = ws.parq; P.offq = ws.offq; P.szq = ws.szq;
     P.cidxq = descent ? ws.cidxq : nullptr;
@@ -940,7 +943,7 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
     if (ev) GB_CUDA_TRY(cudaEventRecord(ev[0], st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.s1, 0, sizeof(uint32_t) * (size_t)B * g.ncomp, st));
     if (descent) GB_CUDA_TRY(cudaMemsetAsync(ws.sz64, 0, sizeof(unsigned long long) * (size_t)B * g.n, st));
-    else GB_CUDA_TRY(cudaMemsetAsync(ws.size, 0, sizeof(uint32_t) * (size_t)B * size_slots(g.n), st));
+    else GB_CUDA_TRY(cudaMemsetAsync(ws.size, 0, sizeof(uint32_t) * (size_t)B * g.n, st));
     k_batch_prep<<<1, kMaxBatch, 0, st>>>(P);
     ++*launches;
     // f.3: a uniform random spanning tree (B = 1), then the caller-tree path

@@ -1,0 +1,14 @@
+# parity (incl. slow full-size C3 subset) + bench variants
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" > gpurun_out/smoke.log 2>&1; echo smoke $?; tail -1 gpurun_out/smoke.log
+timeout 1200 python -m pytest tests/test_gpu_parity.py -m gpu -x -q -k "not c5" > gpurun_out/pytest_gpu.log 2>&1; echo pytest $?
+tail -4 gpurun_out/pytest_gpu.log
+run() { timeout 300 python bench.py --no-cpu-baseline --no-e2e $@ > gpurun_out/b.log 2>&1
+  python -c "
+import json,sys; d=json.loads(open('gpurun_out/b.log').read().strip().splitlines()[-1]); print('$*', round(d['value']/1e9,3), round(d['ms_per_step'],2), {k:round(v,2) for k,v in d['phase_ms_per_step'].items()})" || tail -3 gpurun_out/b.log; }
+run --config c3
+run --config c3 --sub 2
+run --config c4 --steps 20
+run --config c2 --steps 50
+run --config c3 --steps 2 --warmup 1 --walk 1
+run --config c3 --steps 2 --warmup 1 --walk 1 --opt desc_linear=1
+run --config c3 --steps 1 --warmup 1 --walk 2
