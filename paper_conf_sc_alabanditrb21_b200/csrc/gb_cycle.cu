@@ -557,6 +557,12 @@ __global__ void k_accumulate_agree(const uint32_t *__restrict__ pp, int ps, cons
         const int32_t C = __ldg(comp_i + v);
         const uint32_t cs = (uint32_t)(__ldg(coff + C + 1) - __ldg(coff + C));
         int32_t d = 0;
+        if (cs == 1) {
+            // a single-vertex component is its own larger side in every tree
+            // (its labels are not stored per tree)
+            agree[__ldg(bord + v)] += 2 * B;
+            continue;
+        }
         for (int b = 0; b < B; b++) {
             const uint32_t ones = __ldg(s1 + (size_t)b * ncomp + C);
             const uint32_t mine = (__ldg(pp + ((size_t)b * n + v) * ps) >> 31) ? ones : cs - ones;

@@ -394,6 +394,19 @@ __global__ void k_comp_big(const int32_t *__restrict__ coff, int64_t nc, unsigne
     if (best) atomicMax(big, best);
 }
 
+__global__ void k_big_flags(const int32_t *__restrict__ coff, int64_t nc, uint32_t *__restrict__ flag) {
+    for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c <= nc;
+         c += (int64_t)gridDim.x * blockDim.x)
+        flag[c] = c < nc && coff[c + 1] - coff[c] >= 2 ? 1u : 0u;
+}
+
+__global__ void k_big_fill(const uint32_t *__restrict__ flag, const uint32_t *__restrict__ pos, int64_t nc,
+                           int32_t *__restrict__ bigc) {
+    for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < nc;
+         c += (int64_t)gridDim.x * blockDim.x)
+        if (flag[c]) bigc[pos[c]] = (int32_t)c;
+}
+
 // work items of the multi-source BFS: chunks of <= kChunk slots of every
 // vertex heavier than kLight (internal ids 0 .. nlight0-1, degree-sorted)
 __global__ void k_item_counts(const uint32_t *__restrict__ brow, int64_t nlight0, uint32_t *__restrict__ cnt) {
@@ -451,6 +464,7 @@ __global__ void k_view_rank(const uint32_t *__restrict__ bord, const uint32_t *_
         const uint32_t d = sdeg[i];
         if (d > (uint32_t)kLight) atomicAdd(counts, 1ull);
         if (d > (uint32_t)kChunk) atomicAdd(counts + 1, 1ull);
+        if (d == 0) atomicAdd(counts + 2, 1ull);
     }
 }
 
@@ -605,13 +619,29 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
         ING_TRY(cudaStreamSynchronize(st));
         g.ncomp = nc;
         g.cbig = (int32_t)(0xFFFFFFFFull - (hb & 0xFFFFFFFFull));
+        // components with >= 2 vertices (every tree roots each of them; a
+        // single-vertex component is its own finished tree)
+        uint32_t *bflag = nullptr, *bpos = nullptr;
+        ING_ALLOC(bflag, kArBigFlag, 2 * nc + 2);
+        bpos = bflag + nc + 1;
+        k_big_flags<<<grid_for(nc + 1, 256, sms), 256, 0, st>>>(g.coff, nc, bflag);
+        ++*launches;
+        rc = exclusive_scan_u32(bflag, bpos, nc + 1, tmp, ntmp, st, launches);
+        if (rc) goto done;
+        ING_ALLOC(g.bigc, kArBigC, nc);
+        k_big_fill<<<grid_for(nc, 256, sms), 256, 0, st>>>(bflag, bpos, nc, g.bigc);
+        ++*launches;
+        uint32_t hbig = 0;
+        ING_TRY(cudaMemcpyAsync(&hbig, bpos + nc, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+        ING_TRY(cudaStreamSynchronize(st));
+        g.nbig = (int64_t)hbig;
     }
     {
         // degree-sorted view: stable radix sort of the degrees (descending),
         // then the view's CSR with internal neighbour ids and original ids
         uint32_t *deg = nullptr, *sdeg = nullptr, *ids = nullptr;
         unsigned long long *cnt2 = nullptr;
-        ING_ALLOC(deg, kArDeg, 3 * n + 8);
+        ING_ALLOC(deg, kArDeg, 3 * n + 12);
         sdeg = deg + n;
         ids = deg + 2 * n;
         cnt2 = (unsigned long long *)(((uintptr_t)(deg + 3 * n) + 7) & ~(uintptr_t)7);
@@ -634,7 +664,7 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
             rc = radix_sort_pairs(deg, sdeg, ids, g.bord, n, dbits, true, sort_tmp, rs_stmp, rs_scan, st, launches);
             if (rc) goto done;
         }
-        ING_TRY(cudaMemsetAsync(cnt2, 0, 2 * sizeof(unsigned long long), st));
+        ING_TRY(cudaMemsetAsync(cnt2, 0, 3 * sizeof(unsigned long long), st));
         k_view_rank<<<grid_for(n, 256, sms), 256, 0, st>>>(g.bord, sdeg, n, g.brank, cnt2);
         ++*launches;
         rc = exclusive_scan_u32(sdeg, g.brow, n, tmp, ntmp, st, launches);
@@ -646,11 +676,12 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
                 g.row_ptr, g.adj, g.brow, g.bord, g.brank, n, slots, g.badj, g.borig);
             ++*launches;
         }
-        unsigned long long hc[2] = {0, 0};
+        unsigned long long hc[3] = {0, 0, 0};
         ING_TRY(cudaMemcpyAsync(hc, cnt2, sizeof(hc), cudaMemcpyDeviceToHost, st));
         ING_TRY(cudaStreamSynchronize(st));
         g.nlight0 = (int64_t)hc[0];
         g.nmulti = (int64_t)hc[1];
+        g.niso = (int64_t)hc[2];          // isolated vertices: internal ids [n - niso, n)
         // work items: chunks of <= kChunk slots of every vertex heavier than kLight
         if (g.nlight0 > 0) {
             k_item_counts<<<grid_for(g.nlight0, 256, sms), 256, 0, st>>>(g.brow, g.nlight0, upc);

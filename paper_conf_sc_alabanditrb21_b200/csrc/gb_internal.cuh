@@ -121,6 +121,9 @@ struct Graph {
     int32_t *coff = nullptr;            // [ncomp+1] component offsets (pre of the root)
     int32_t *cverts = nullptr;          // [n] vertices grouped by component, ascending
     int32_t cbig = 0;                   // largest component
+    int32_t *bigc = nullptr;            // [nbig] components with >= 2 vertices
+    int64_t nbig = 0;
+    int64_t niso = 0;                   // isolated vertices (internal ids [n - niso, n))
     // Degree-sorted view for the multi-source BFS (gb_msbfs.cu): internal ids
     // 0..n-1 order the vertices by degree, descending (ties by original id),
     // so a warp's 32 consecutive vertices have similar degrees and the hubs
@@ -248,7 +251,7 @@ enum ArenaSlot {
     kArRowPtr64, kArCol, kArSign, kArErr, kArRowPtr, kArAdj, kArAdjEid, kArEdges, kArComp,
     kArCverts, kArUptr, kArUpc, kArEbase, kArScanTmp, kArLab, kArFlag, kArRank, kArCoff,
     kArBrow, kArBadj, kArBorig, kArBord, kArBrank, kArItems, kArDeg, kArSortTmp, kArCkeys,
-    kArEdgesI, kArCompI, kArRsScan, kArSlots
+    kArEdgesI, kArCompI, kArRsScan, kArBigFlag, kArBigC, kArSlots
 };
 void *arena(int slot, size_t bytes);   // nullptr on allocation failure (error set)
 void arena_free_all();

@@ -44,7 +44,8 @@ constexpr int kMsMaxBlocks = 2048;   // capacity of the per-block count table
 struct MsParams {
     const uint32_t *brow, *badj, *borig, *bord, *brank;
     const uint2 *items;
-    const int32_t *coff, *cverts;
+    const int32_t *coff, *cverts, *bigc, *comp_i;
+    int64_t nbig, niso;
     int64_t n, ncomp, nitems, nmulti_items, nlight0, nmulti, ls, nwords, itemwords;
     int B;
     unsigned long long full;
@@ -428,11 +429,30 @@ __device__ __forceinline__ int select_bit64(unsigned long long m, int r) {
 // (ascending)[rkey(b, C) mod |C|]; level 0 of every tree
 // ---------------------------------------------------------------------------
 __global__ void k_ms_roots(MsParams P) {
-    const int64_t total = (int64_t)P.B * P.ncomp;
+    // single-vertex components (the isolated vertices, internal ids
+    // [n - niso, n)): their one-vertex trees are identical in every tree --
+    // reached in all trees at level 0, never on a frontier, labels pre =
+    // coff[C], pi = 0, size 1 (read from the component table wherever needed)
+    for (int64_t i = P.n - P.niso + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        P.vis[i] = P.full;
+        if (!P.irec) {
+            // layout 1 (walks 1, 2, option jump) reads pre-indexed records of
+            // every vertex: the one-vertex trees' records, per tree
+            const uint32_t pre = (uint32_t)P.coff[P.comp_i[i]];
+            for (int b = 0; b < P.B; b++) {
+                const size_t nb = (size_t)b * P.n;
+                P.pp[nb + i] = pre;
+                P.rec[nb + pre] = make_uint2(pre, 1u);
+                if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
+            }
+        }
+    }
+    const int64_t total = (int64_t)P.B * P.nbig;
     for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
          x += (int64_t)gridDim.x * blockDim.x) {
-        const int b = (int)(x / P.ncomp);
-        const int64_t C = x - (int64_t)b * P.ncomp;
+        const int b = (int)(x / P.nbig);
+        const int64_t C = P.bigc[x - (int64_t)b * P.nbig];
         const uint32_t sz = (uint32_t)(P.coff[C + 1] - P.coff[C]);
         const uint64_t rk = root_key(P.tkey[b], C);
         const uint32_t r = (uint32_t)P.cverts[P.coff[C] + (int64_t)(rk % sz)];
@@ -440,18 +460,6 @@ __global__ void k_ms_roots(MsParams P) {
         const unsigned long long bit = 1ull << b;
         atomicOr(P.vis + ri, bit);
         const size_t nb = (size_t)b * P.n;
-        if (P.brow[ri + 1] == P.brow[ri]) {
-            // isolated vertex: a one-vertex tree, finished here (pi = 0)
-            const uint32_t pre = (uint32_t)P.coff[C];
-            if (P.irec) {
-                P.irec[nb + ri] = make_uint4(ri, pre, 1u, 0u);
-            } else {
-                P.pp[nb + ri] = pre;
-                P.rec[nb + pre] = make_uint2(pre, 1u);
-                if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
-            }
-            continue;
-        }
         const unsigned long long old = atomicAdd((unsigned long long *)(P.lvl + b * P.ls), 1ull << 32);
         const uint32_t pos = (uint32_t)(old >> 32);
         P.qv[nb + pos] = ri;
@@ -822,6 +830,7 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
     MsParams P;
     P.brow = g.brow; P.badj = g.badj; P.borig = g.borig; P.bord = g.bord; P.brank = g.brank;
     P.items = g.items; P.coff = g.coff; P.cverts = g.cverts;
+    P.bigc = g.bigc; P.nbig = g.nbig; P.niso = g.niso; P.comp_i = g.comp_i;
     P.n = g.n; P.ncomp = g.ncomp; P.nitems = g.nitems; P.nmulti_items = g.nmulti_items;
     P.nlight0 = g.nlight0; P.nmulti = g.nmulti; P.ls = g.n + 2;
     P.nwords = (g.n + 31) / 32;
@@ -841,7 +850,7 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
     GB_CUDA_TRY(cudaMemsetAsync(ws.fr, 0, sizeof(unsigned long long) * (size_t)g.n, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.fbm, 0, sizeof(uint32_t) * 6 * (size_t)P.nwords, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.msflag, 0, sizeof(int32_t) * 8, st));
-    const int64_t work = (int64_t)B * g.ncomp;
+    const int64_t work = std::max<int64_t>((int64_t)B * g.nbig, g.niso);
     k_ms_roots<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, 8192)), 256, 0, st>>>(P);
     ++*launches;
     void *args[] = {&P};

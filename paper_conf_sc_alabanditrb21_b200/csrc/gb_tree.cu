@@ -36,6 +36,7 @@ namespace cg = cooperative_groups;
 struct TreeParams {
     const uint32_t *row_ptr, *adj;             // original CSR (push BFS of caller trees)
     const uint32_t *brank, *bord;              // original <-> internal ids
+    const uint32_t *brow;                      // degree-sorted view rows (isolated vertices)
     const int32_t *comp, *comp_i, *coff, *cverts;
     int64_t n, ncomp, nw;  // nw = state words per tree ((n + 3) / 4)
     int32_t cbig;
@@ -825,6 +826,12 @@ __global__ void k_debug_tree(TreeParams P, int32_t *parent, int32_t *dist, int32
         const uint32_t v = P.bord[i];   // labels live in internal ids; outputs by original id
         parent[v] = -1;
         dist[v] = 0;
+        if (P.brow[i + 1] == P.brow[i]) {
+            // isolated vertex: a one-vertex tree (labels not stored per tree)
+            size[v] = 1;
+            pre[v] = P.coff[P.comp_i[i]];
+            continue;
+        }
         size[v] = 1 + (P.sz64 ? (int32_t)(uint32_t)P.sz64[i] : (int32_t)P.size[szi(P, (uint32_t)i)]);
         pre[v] = (int32_t)((P.irec ? P.irec[i].y : P.pp[i]) & kIdMask);
     }
@@ -870,7 +877,7 @@ static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_
                               bool descent, int b0 = 0) {
     TreeParams P;
     P.row_ptr = g.row_ptr; P.adj = g.adj;
-    P.brank = g.brank; P.bord = g.bord;
+    P.brank = g.brank; P.bord = g.bord; P.brow = g.brow;
     P.comp = g.comp; P.comp_i = g.comp_i; P.coff = g.coff; P.cverts = g.cverts;
     P.n = g.n; P.ncomp = g.ncomp; P.nw = (g.n + 3) / 4; P.cbig = g.cbig;
     P.B = B; P.ls = g.n + 2;
