@@ -91,7 +91,9 @@ struct State {
     bool ws_irec = false;
     cudaStream_t stream = nullptr;
     int32_t *d_cnt = nullptr, *d_agree = nullptr;  // gb_balance's device counters
+    int64_t cnt_cap_m = 0, cnt_cap_n = 0;          // their capacities (edges, vertices)
     int32_t *d_given = nullptr;                    // caller tree (gb_balance_given_tree)
+    int64_t given_cap = 0;
     unsigned long long *d_visited = nullptr;       // [kMaxBatch]
     unsigned long long *d_rec_stats = nullptr;     // [kRecCap][4]
     unsigned long long *d_tot = nullptr;           // [4] sum k, cycles, max depth over every tree of the call
@@ -562,13 +564,19 @@ int gb_selftest(void) {
 // release the loaded graph and everything sized by it, but keep the stream,
 // the statistics buffer and (if asked) the tree workspace for a reload
 static void release_graph(bool keep_ws) {
-    if (!keep_ws) free_ws(S.ws);
+    if (!keep_ws) {
+        free_ws(S.ws);
+        // gb_balance's counters and the caller-tree buffer are sized by the
+        // graph; a reload of the same shape keeps them (cudaFree synchronises)
+        if (S.d_cnt) cudaFree(S.d_cnt);
+        if (S.d_agree) cudaFree(S.d_agree);
+        if (S.d_given) cudaFree(S.d_given);
+        S.d_cnt = S.d_agree = nullptr;
+        S.d_given = nullptr;
+        S.given_cap = 0;
+        S.cnt_cap_m = S.cnt_cap_n = 0;
+    }
     free_graph(S.g);
-    if (S.d_cnt) cudaFree(S.d_cnt);
-    if (S.d_agree) cudaFree(S.d_agree);
-    if (S.d_given) cudaFree(S.d_given);
-    S.d_cnt = S.d_agree = nullptr;
-    S.d_given = nullptr;
     S.loaded = false;
     S.h_comp.clear();
 }
@@ -724,9 +732,15 @@ int gb_balance(int64_t num_trees, uint64_t seed, uint32_t *out_edge_flip_counts,
     if (!S.loaded) { set_error("no graph loaded"); return GB_ESTATE; }
     if (num_trees < 0 || num_trees > (1ll << 30) - 1) { set_error("num_trees out of range"); return GB_EINVAL; }
     if ((S.g.m > 0 && !out_edge_flip_counts) || !out_vertex_agree) { set_error("NULL output"); return GB_EINVAL; }
-    if (!S.d_cnt) {
+    if (!S.d_cnt || S.cnt_cap_m < std::max<int64_t>(S.g.m, 1) || S.cnt_cap_n < S.g.n) {
+        if (S.d_cnt) cudaFree(S.d_cnt);
+        if (S.d_agree) cudaFree(S.d_agree);
+        S.d_cnt = S.d_agree = nullptr;
+        S.cnt_cap_m = S.cnt_cap_n = 0;
         GB_CUDA_TRY(cudaMalloc(&S.d_cnt, sizeof(int32_t) * std::max<int64_t>(S.g.m, 1)));
         GB_CUDA_TRY(cudaMalloc(&S.d_agree, sizeof(int32_t) * S.g.n));
+        S.cnt_cap_m = std::max<int64_t>(S.g.m, 1);
+        S.cnt_cap_n = S.g.n;
     }
     GB_CUDA_TRY(cudaMemsetAsync(S.d_cnt, 0, sizeof(int32_t) * std::max<int64_t>(S.g.m, 1), S.stream));
     GB_CUDA_TRY(cudaMemsetAsync(S.d_agree, 0, sizeof(int32_t) * S.g.n, S.stream));
@@ -783,7 +797,13 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip, uint64_t *sum_cy
     }
     for (int64_t c = 0; c < S.g.ncomp; c++)
         if (roots[c] != 1) { set_error("need exactly one root (-1) per connected component"); return GB_EINVAL; }
-    if (!S.d_given) GB_CUDA_TRY(cudaMalloc(&S.d_given, sizeof(int32_t) * n));
+    if (!S.d_given || S.given_cap < n) {
+        if (S.d_given) cudaFree(S.d_given);
+        S.d_given = nullptr;
+        S.given_cap = 0;
+        GB_CUDA_TRY(cudaMalloc(&S.d_given, sizeof(int32_t) * n));
+        S.given_cap = n;
+    }
     GB_CUDA_TRY(cudaMemcpy(S.d_given, parent, sizeof(int32_t) * n, cudaMemcpyHostToDevice));
     int rc = run_single_tree(0, 0, S.d_given);
     if (rc) return rc;

@@ -312,10 +312,12 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
                 const unsigned long long key = parent_key(tk, o & kIdMask, o_w, o >> 31);
                 if (key < best) { best = key; bk = k; }
             }
-            const unsigned long long bit = 1ull << t;
-            if (bk & 1) atomicOr(&W.pk[0][src], bit);
-            if (bk & 2) atomicOr(&W.pk[1][src], bit);
-            if (bk & 4) atomicOr(&W.pk[2][src], bit);
+            // 32-bit shared atomics on the plane half holding bit t (the
+            // 64-bit ones compile to compare-and-swap loops)
+            const uint32_t bit = 1u << (t & 31), half = (uint32_t)t >> 5;
+            if (bk & 1) atomicOr(reinterpret_cast<uint32_t *>(&W.pk[0][src]) + half, bit);
+            if (bk & 2) atomicOr(reinterpret_cast<uint32_t *>(&W.pk[1][src]) + half, bit);
+            if (bk & 4) atomicOr(reinterpret_cast<uint32_t *>(&W.pk[2][src]) + half, bit);
         }
         __syncwarp();
     }
