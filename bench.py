@@ -371,8 +371,11 @@ def main():
     peak, peak_src = load_peaks()
     achieved = dom_bytes_per_launch / (dom_ms_per_launch / 1000.0) / 1e9
     bfs_kernel = "k_tbfs" if any(kv.replace(" ", "") == "bfs=0" for kv in args.opt) else "k_msbfs"
+    opts = {kv.replace(" ", "").split("=")[0]: kv.replace(" ", "").split("=")[1] for kv in args.opt}
+    walk_kernel = {0: "k_cycles_irec" if opts.get("jump", "1") == "1" else "k_cycles_jump",
+                   1: "k_cycles_descent", 2: "k_cycles_paper"}[args.walk]
     kernel_of = {"bfs": bfs_kernel, "bottom_up": "k_bottom_up", "top_down": "k_top_down",
-                 "cycles": "k_cycles_two_ended", "accumulate": "k_accumulate_edges", "init": "k_tb_roots"}
+                 "cycles": walk_kernel, "accumulate": "k_accumulate_edges", "init": "k_ms_roots"}
     traffic = ncu_traffic(args.config, kernel_of[dom], trees_in_step / dom_launches)
     path_bytes = sum(bytes_per_tree.values()) * total_trees * args.steps / world
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak, "unit": "GB/s",

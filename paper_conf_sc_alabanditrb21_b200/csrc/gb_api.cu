@@ -168,9 +168,9 @@ static int ensure_workspace(int B, bool descent) {
     ALLOC(w.qr, n);
     ALLOC(w.pkeyq, n);
     // multi-source BFS state (one bit per tree)
-    ALLOC(w.vis, n);
-    ALLOC(w.fr, 2 * n);
-    ALLOC(w.hacc, std::max<int64_t>(g.nmulti, 1));
+    ALLOC(w.vis, 2 * n);
+    ALLOC(w.fr, 4 * n);
+    ALLOC(w.hacc, 2 * std::max<int64_t>(g.nmulti, 1));
     ALLOC(w.hbest, std::max<int64_t>(g.nmulti, 1) * kMsBatch);
     ALLOC(w.msflag, 8);
     ALLOC(w.mscnt, (int64_t)kMsBatch * 2048);
@@ -289,7 +289,7 @@ __global__ void k_cloud_states(const unsigned long long *rec, int64_t k, unsigne
 
 static int auto_batch(int64_t ntrees) {
     if (S.opt.sampler != 0) return 1;   // sampled trees go one at a time (caller-tree path)
-    // the multi-source BFS holds one bit per tree in a 64-bit word
+    // the multi-source BFS holds one bit per tree in a 128-bit word
     if (S.opt.batch > 0) return (int)std::min<int64_t>(S.opt.batch, kMsBatch);
     const size_t have = S.free_at_load;
     int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk >= 1));
@@ -418,7 +418,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
         k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, nb, seed, t0, stride);
         ++T.launches;
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 3 * nb, st));
-        GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
+        GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * 2 * std::max<int64_t>(S.g.nmulti, 1), st));
         GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
         const int32_t *given = nullptr;
         if (S.opt.sampler == 2 || (S.opt.sampler == 1 && !S.opt.wilson)) {
@@ -491,7 +491,7 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
     k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, 1, seed, t, 1);
     ++T.launches;
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.tstat, 0, sizeof(unsigned long long) * 3, st));
-    GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1), st));
+    GB_CUDA_TRY(cudaMemsetAsync(S.ws.hacc, 0, sizeof(unsigned long long) * 2 * std::max<int64_t>(S.g.nmulti, 1), st));
     GB_CUDA_TRY(cudaMemsetAsync(S.ws.hbest, 0xFF, sizeof(unsigned long long) * std::max<int64_t>(S.g.nmulti, 1) * kMsBatch, st));
     const bool user_tree = d_given != nullptr;
     if (!d_given && (S.opt.sampler == 2 || (S.opt.sampler == 1 && !S.opt.wilson))) {

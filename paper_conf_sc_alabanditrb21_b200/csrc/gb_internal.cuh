@@ -15,7 +15,7 @@ constexpr int32_t kInf = 0x7F7F7F7F;         // "unvisited" BFS distance (memset
 constexpr uint32_t kNone = 0xFFFFFFFFu;
 constexpr int kMaxBatch = 128;               // trees per batch (smem tables)
 constexpr int kBlock = 256;                  // threads per CTA of the cooperative kernels
-constexpr int kMsBatch = 64;                 // trees per multi-source BFS (one bit each)
+constexpr int kMsBatch = 128;                // trees per multi-source BFS (one bit each, two 64-bit halves)
 constexpr int kLight = 8;                    // BFS: degree <= kLight -> one lane per vertex
 constexpr int kChunk = 256;                  // BFS: slots per warp work item of a heavier vertex
 constexpr int kTbMax = 16;                   // tree-parallel BFS: trees per launch (per-tree bitmaps)
@@ -179,13 +179,13 @@ struct Workspace {
     uint2 *jrec = nullptr;     // [G][n][K] K-level ancestor records of one cycle group (option "jump")
     int jrec_cap = 0;          // G * K the buffer holds
     // multi-source BFS state (one bit per tree of the batch, internal ids)
-    unsigned long long *vis = nullptr;  // [n] trees that reached the vertex
-    unsigned long long *fr = nullptr;   // [2][n] frontier of level L / L+1
-    unsigned long long *hacc = nullptr; // [nmulti] discoveries of multi-chunk vertices
-    unsigned long long *hbest = nullptr;// [nmulti][64] their best parent keys
+    unsigned long long *vis = nullptr;  // [n][2] trees that reached the vertex (two 64-tree halves)
+    unsigned long long *fr = nullptr;   // [2][n][2] frontier of level L / L+1
+    unsigned long long *hacc = nullptr; // [nmulti][2] discoveries of multi-chunk vertices
+    unsigned long long *hbest = nullptr;// [nmulti][128] their best parent keys
     int32_t *msflag = nullptr;          // [8]: [0..1] a multi-chunk vertex discovered something,
                                         // [4..6] frontier sizes (levels mod 3)
-    uint32_t *mscnt = nullptr;          // [64][2048] per-block discovery counts
+    uint32_t *mscnt = nullptr;          // [128][2048] per-block discovery counts
     unsigned long long *msprof = nullptr;  // [256][4] BFS phase timestamps (option "msprof")
     // tree-parallel BFS state (gb_tbfs.cu), G <= kTbMax trees per launch
     uint32_t *tbm = nullptr;            // [G][6][ceil(n/32)] per-tree bitmaps + [ceil(n/32)] "finished"

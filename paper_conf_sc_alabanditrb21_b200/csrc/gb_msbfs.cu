@@ -1,11 +1,11 @@
-// gb_msbfs.cu -- §8 rows a.2 + a.3 for a batch of B <= 64 sampled trees at
+// gb_msbfs.cu -- §8 rows a.2 + a.3 for a batch of B <= 128 sampled trees at
 // once: hashed roots, level-synchronous BFS and min-hash parent selection.
 //
 // The paper builds one BFS tree at a time (§3.1, Fig. 11 "spanning tree"
 // 6 %) and rejects one-tree-per-thread for memory and locality on a 12 GB
 // Titan V (L250).  Here the B trees of a batch share every pass over the
-// graph (§8 a.9, multi-source BFS): each vertex carries a 64-bit word with
-// one bit per tree --
+// graph (§8 a.9, multi-source BFS): each vertex carries a 128-bit word with
+// one bit per tree (two 64-bit halves, interleaved: trees 0-63, 64-127) --
 //   vis[v]  trees that have reached v,
 //   F_L[v]  trees in which v is on level L (the frontier),
 // plus two bitmaps with one bit per vertex: "F_L[v] != 0" (the frontier
@@ -48,15 +48,15 @@ struct MsParams {
     int64_t nbig, niso;
     int64_t n, ncomp, nitems, nmulti_items, nlight0, nmulti, ls, nwords, itemwords;
     int B;
-    unsigned long long full;
-    unsigned long long *vis, *fr, *hacc, *hbest;
+    unsigned long long full0, full1;   // the "every tree" masks of the two halves
+    unsigned long long *vis, *fr, *hacc, *hbest;   // vis, fr, hacc: [n][2] (half h at 2u + h); hbest [nmulti][128]
     uint32_t *fbm;     // [3][nwords] frontier bitmaps (level L % 3)
     uint32_t *fullbm;  // [nwords] finished vertices
     uint32_t *tb;      // [2][nwords] "has a neighbour on the frontier" (push levels)
     uint32_t *fcnt;    // [3] vertices on the frontier of level L (mod 3); [3] vertices finished
     int64_t push_div;  // a level pushes first while frontier * push_div <= unfinished vertices
     int32_t *flag;
-    uint32_t *mscnt;   // [64][kMsMaxBlocks] discoveries per tree per block (phase A)
+    uint32_t *mscnt;   // [128][kMsMaxBlocks] discoveries per tree per block (phase A)
     const uint64_t *tkey;
     uint32_t *qv, *parq, *pp;
     uint2 *rec, *crec;
@@ -100,10 +100,29 @@ __device__ __forceinline__ bool bm_test(const uint32_t *bm, uint32_t u) {
     return (__ldcg(bm + (u >> 5)) >> (u & 31)) & 1u;
 }
 
-// frontier word of u (0 unless u is on the current level in some tree)
+// the two halves of a vertex's 128-bit tree mask
+struct W2 {
+    unsigned long long a, b;   // trees 0-63, 64-127
+};
+__device__ __forceinline__ W2 ld2(const unsigned long long *p) {
+    const uint4 v = __ldcg(reinterpret_cast<const uint4 *>(p));
+    return W2{(unsigned long long)v.x | ((unsigned long long)v.y << 32),
+              (unsigned long long)v.z | ((unsigned long long)v.w << 32)};
+}
+__device__ __forceinline__ void st2(unsigned long long *p, W2 w) {
+    *reinterpret_cast<uint4 *>(p) = make_uint4((uint32_t)w.a, (uint32_t)(w.a >> 32), (uint32_t)w.b,
+                                               (uint32_t)(w.b >> 32));
+}
+
+// half h of the frontier word of u (0 unless u is on the current level in
+// some tree)
 __device__ __forceinline__ unsigned long long fr_word(const unsigned long long *F, const uint32_t *bm,
-                                                      uint32_t u) {
-    return bm_test(bm, u) ? __ldcg(F + u) : 0ull;
+                                                      uint32_t u, int h) {
+    return bm_test(bm, u) ? __ldcg(F + 2 * (size_t)u + h) : 0ull;
+}
+// both halves (one 16-byte load)
+__device__ __forceinline__ W2 fr_word2(const unsigned long long *F, const uint32_t *bm, uint32_t u) {
+    return bm_test(bm, u) ? ld2(F + 2 * (size_t)u) : W2{0ull, 0ull};
 }
 
 // level-(L+1) entry `pos` of tree t: the vertex and its parent | neg << 31,
@@ -125,18 +144,25 @@ __device__ __forceinline__ void ms_emit_par(const MsParams &P, int t, uint32_t p
 }
 
 // OR of the frontier words over the slots [s0, s1) (one warp, lanes stride)
-__device__ __forceinline__ unsigned long long ms_chunk_or(const MsParams &P, const unsigned long long *F,
-                                                          const uint32_t *bm, uint32_t s0, uint32_t s1) {
+__device__ __forceinline__ W2 ms_chunk_or(const MsParams &P, const unsigned long long *F,
+                                          const uint32_t *bm, uint32_t s0, uint32_t s1) {
     const int lane = threadIdx.x & 31;
-    unsigned long long acc = 0;
+    W2 acc{0ull, 0ull};
     uint32_t j = s0 + lane;
     for (; j + 96 < s1; j += 128) {
         const uint32_t a0 = __ldg(P.badj + j) & kIdMask, a1 = __ldg(P.badj + j + 32) & kIdMask;
         const uint32_t a2 = __ldg(P.badj + j + 64) & kIdMask, a3 = __ldg(P.badj + j + 96) & kIdMask;
-        acc |= fr_word(F, bm, a0) | fr_word(F, bm, a1) | fr_word(F, bm, a2) | fr_word(F, bm, a3);
+        const W2 w0 = fr_word2(F, bm, a0), w1 = fr_word2(F, bm, a1);
+        const W2 w2 = fr_word2(F, bm, a2), w3 = fr_word2(F, bm, a3);
+        acc.a |= w0.a | w1.a | w2.a | w3.a;
+        acc.b |= w0.b | w1.b | w2.b | w3.b;
     }
-    for (; j < s1; j += 32) acc |= fr_word(F, bm, __ldg(P.badj + j) & kIdMask);
-    return warp_or64(acc);
+    for (; j < s1; j += 32) {
+        const W2 w = fr_word2(F, bm, __ldg(P.badj + j) & kIdMask);
+        acc.a |= w.a;
+        acc.b |= w.b;
+    }
+    return W2{warp_or64(acc.a), warp_or64(acc.b)};
 }
 
 __device__ __forceinline__ unsigned long long warp_min64(unsigned long long v) {
@@ -155,7 +181,8 @@ __device__ __forceinline__ unsigned long long warp_min64(unsigned long long v) {
 __device__ __forceinline__ void ms_chunk_keys(const MsParams &P, const unsigned long long *F,
                                               const uint32_t *bm, uint32_t s0, uint32_t s1,
                                               unsigned long long want, uint32_t ow, const uint64_t *s_tk,
-                                              bool whole, unsigned long long &b0, unsigned long long &b1) {
+                                              bool whole, unsigned long long &b0, unsigned long long &b1,
+                                              int h) {
     const int lane = threadIdx.x & 31;
     b0 = ~0ull;
     b1 = ~0ull;
@@ -166,7 +193,7 @@ __device__ __forceinline__ void ms_chunk_keys(const MsParams &P, const unsigned 
         unsigned long long f = 0;
         if (j < s1) {
             const uint32_t a = __ldg(P.badj + j);
-            f = fr_word(F, bm, a & kIdMask) & want;
+            f = fr_word(F, bm, a & kIdMask, h) & want;
             if (f) o = __ldg(P.borig + j) | (a & kNegBit);
         }
         for (unsigned long long rem = warp_or64(f); rem; rem &= rem - 1) {
@@ -197,7 +224,7 @@ struct WarpScratch {
     uint32_t lo[kLight][32];             // candidate neighbour (original id) | neg << 31 (hashing)
     uint32_t li[kLight][32];             // the same neighbour as an internal id | neg << 31 (output)
     uint32_t ow[32];                     // original id of each lane's vertex
-    unsigned long long best[kMsBatch];   // item parents: best key per tree
+    unsigned long long best[64];         // item parents: best key per tree (of the half)
 };
 constexpr size_t kMsSmem = sizeof(WarpScratch) * kMsWarps;
 
@@ -231,16 +258,20 @@ __device__ __forceinline__ uint32_t transpose32(uint32_t x) {
 // words (vertex x tree bits) are transposed so that lane t holds, for trees
 // t and t + 32, the mask of vertices to append; it reserves its run of the
 // tree's level list with one shared-memory add and writes its entries.
+// Half h of the 128 trees (trees 64h .. 64h + 63; s_tk, s_base and s_pos
+// point at the half's first tree).
 __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsigned long long *F,
                                                  const unsigned long long *Nx, const uint32_t *bm,
                                                  uint32_t i, bool act, const uint64_t *s_tk,
-                                                 const uint32_t *s_base, uint32_t *s_pos, WarpScratch &W) {
+                                                 const uint32_t *s_base, uint32_t *s_pos, WarpScratch &W,
+                                                 int half) {
     const int lane = threadIdx.x & 31;
     unsigned long long nw = 0, s2m = 0;   // discovered trees / those with >= 2 candidates
     unsigned long long c[kLight];
     uint32_t ow = 0;
+    if (act) nw = __ldcg(Nx + 2 * (size_t)i + half);
+    if (!__any_sync(0xFFFFFFFFu, nw != 0)) return;   // nothing in this half
     if (act) {
-        nw = __ldcg(Nx + i);
         const uint32_t rs = __ldg(P.brow + i);
         const uint32_t deg = __ldg(P.brow + i + 1) - rs;
         ow = __ldg(P.bord + i);
@@ -250,7 +281,7 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
             c[k] = 0;
             if (k < (int)deg) {
                 const uint32_t a = __ldg(P.badj + rs + k);
-                c[k] = fr_word(F, bm, a & kIdMask) & nw;
+                c[k] = fr_word(F, bm, a & kIdMask, half) & nw;
                 if (c[k]) {
                     W.lo[k][lane] = __ldg(P.borig + rs + k) | (a & kNegBit);
                     W.li[k][lane] = a;
@@ -343,7 +374,7 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
             if ((mask >> lane) & 1u) {
                 const uint32_t k = (uint32_t)((mine_pk0 >> t) & 1ull) | ((uint32_t)((mine_pk1 >> t) & 1ull) << 1) |
                                    ((uint32_t)((mine_pk2 >> t) & 1ull) << 2);
-                const size_t o = (size_t)t * P.n + base + __popc(mask & lt);
+                const size_t o = (size_t)(t + 64 * half) * P.n + base + __popc(mask & lt);
                 P.qv[o] = i;
                 P.parq[o] = W.li[k][lane];
             }
@@ -360,7 +391,7 @@ __device__ __forceinline__ void ms_item_parents(const MsParams &P, const unsigne
                                                 const uint32_t *bm, uint32_t s0, uint32_t s1,
                                                 unsigned long long want, uint32_t ow,
                                                 const uint64_t *s_tk, WarpScratch &W,
-                                                uint32_t &p0, uint32_t &p1) {
+                                                uint32_t &p0, uint32_t &p1, int h) {
     const int lane = threadIdx.x & 31;
     uint16_t *pl = reinterpret_cast<uint16_t *>(W.ml);   // <= 32 * 64 pairs fit kMultiCap * 2
     const uint32_t j = s0 + lane;
@@ -368,7 +399,7 @@ __device__ __forceinline__ void ms_item_parents(const MsParams &P, const unsigne
     uint32_t o = 0;
     if (j < s1) {
         const uint32_t a = __ldg(P.badj + j);
-        f = fr_word(F, bm, a & kIdMask) & want;
+        f = fr_word(F, bm, a & kIdMask, h) & want;
         if (f) o = __ldg(P.borig + j) | (a & kNegBit);
     }
     unsigned long long s1m = f, s2m = 0;   // trees with >= 1 / >= 2 candidates
@@ -437,7 +468,7 @@ __global__ void k_ms_roots(MsParams P) {
     // coff[C], pi = 0, size 1 (read from the component table wherever needed)
     for (int64_t i = P.n - P.niso + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.n;
          i += (int64_t)gridDim.x * blockDim.x) {
-        P.vis[i] = P.full;
+        st2(P.vis + 2 * i, W2{P.full0, P.full1});
         if (!P.irec) {
             // layout 1 (walks 1, 2, option jump) reads pre-indexed records of
             // every vertex: the one-vertex trees' records, per tree
@@ -459,14 +490,15 @@ __global__ void k_ms_roots(MsParams P) {
         const uint64_t rk = root_key(P.tkey[b], C);
         const uint32_t r = (uint32_t)P.cverts[P.coff[C] + (int64_t)(rk % sz)];
         const uint32_t ri = P.brank[r];
-        const unsigned long long bit = 1ull << b;
-        atomicOr(P.vis + ri, bit);
+        const unsigned long long bit = 1ull << (b & 63);
+        const int h = b >> 6;
+        atomicOr(P.vis + 2 * (size_t)ri + h, bit);
         const size_t nb = (size_t)b * P.n;
         const unsigned long long old = atomicAdd((unsigned long long *)(P.lvl + b * P.ls), 1ull << 32);
         const uint32_t pos = (uint32_t)(old >> 32);
         P.qv[nb + pos] = ri;
         P.parq[nb + pos] = ri;
-        atomicOr(P.fr + ri, bit);
+        atomicOr(P.fr + 2 * (size_t)ri + h, bit);
         atomicOr(P.fbm + (ri >> 5), 1u << (ri & 31));
     }
 }
@@ -514,12 +546,12 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
     const int64_t l0 = P.nlight0 & ~31ll;   // light tiles start word-aligned
     const int64_t nl_tiles = (P.n - l0 + kBlock - 1) / kBlock;
     const int64_t ntiles = nit_tiles + nl_tiles;
-    const unsigned long long full = P.full;
+    const W2 full{P.full0, P.full1};
     const uint32_t nblk = gridDim.x;
     __shared__ uint32_t s_fc, s_ff;
     for (int L = 0;; L++) {
-        const unsigned long long *F = P.fr + (size_t)(L & 1) * P.n;
-        unsigned long long *Nx = P.fr + (size_t)((L + 1) & 1) * P.n;
+        const unsigned long long *F = P.fr + (size_t)(L & 1) * 2 * P.n;
+        unsigned long long *Nx = P.fr + (size_t)((L + 1) & 1) * 2 * P.n;
         const uint32_t *bm = P.fbm + (size_t)(L % 3) * P.nwords;
         uint32_t *nbm = P.fbm + (size_t)((L + 1) % 3) * P.nwords;
         uint32_t *cbm = P.fbm + (size_t)((L + 2) % 3) * P.nwords;   // free: cleared for L+2
@@ -579,25 +611,31 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                     if (push && !bm_test(tbc, i)) continue;
                     const uint32_t s1 = min(s0 + (uint32_t)kChunk, __ldg(P.brow + i + 1));
                     const bool multi = k < P.nmulti_items;
-                    const unsigned long long vis = __ldcg(P.vis + i);
-                    const unsigned long long part = ms_chunk_or(P, F, bm, s0, s1) & ~vis;
+                    const W2 vis = ld2(P.vis + 2 * (size_t)i);
+                    W2 part = ms_chunk_or(P, F, bm, s0, s1);
+                    part.a &= ~vis.a;
+                    part.b &= ~vis.b;
                     if (multi) {
-                        if (part && lane == 0) {
-                            atomicOr(P.hacc + i, part);
+                        if ((part.a | part.b) && lane == 0) {
+                            if (part.a) atomicOr(P.hacc + 2 * (size_t)i, part.a);
+                            if (part.b) atomicOr(P.hacc + 2 * (size_t)i + 1, part.b);
                             P.flag[L & 1] = 1;
                         }
-                    } else if (part) {
+                    } else if (part.a | part.b) {
                         if (lane == 0) {
-                            Nx[i] = part;
-                            P.vis[i] = vis | part;
+                            st2(Nx + 2 * (size_t)i, part);
+                            const W2 nv{vis.a | part.a, vis.b | part.b};
+                            st2(P.vis + 2 * (size_t)i, nv);
                             atomicOr(nbm + (i >> 5), 1u << (i & 31));
-                            if ((vis | part) == full) {
+                            if (nv.a == full.a && nv.b == full.b) {
                                 atomicOr(P.fullbm + (i >> 5), 1u << (i & 31));
                                 atomicAdd(&s_ff, 1u);
                             }
                         }
-                        if ((part >> lane) & 1ull) atomicAdd(&s_cnt[lane], 1u);
-                        if ((part >> (lane + 32)) & 1ull) atomicAdd(&s_cnt[lane + 32], 1u);
+                        if ((part.a >> lane) & 1ull) atomicAdd(&s_cnt[lane], 1u);
+                        if ((part.a >> (lane + 32)) & 1ull) atomicAdd(&s_cnt[lane + 32], 1u);
+                        if ((part.b >> lane) & 1ull) atomicAdd(&s_cnt[lane + 64], 1u);
+                        if ((part.b >> (lane + 32)) & 1ull) atomicAdd(&s_cnt[lane + 96], 1u);
                         if (lane == 0) atomicAdd(&s_fc, 1u);
                     }
                 }
@@ -608,33 +646,42 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                 const bool mine = (int64_t)i < P.n && (int64_t)i >= P.nlight0;
                 const uint32_t fw = __ldcg(P.fullbm + (v0 >> 5));
                 const uint32_t tw = push ? __ldcg(tbc + (v0 >> 5)) : ~0u;
-                unsigned long long nw = 0;
+                W2 nw{0ull, 0ull};
                 bool nowfull = false;
                 if (mine && !((fw >> lane) & 1u) && ((tw >> lane) & 1u)) {
-                    const unsigned long long vis = __ldcg(P.vis + i);
+                    const W2 vis = ld2(P.vis + 2 * (size_t)i);
                     const uint32_t rs = __ldg(P.brow + i);
                     const uint32_t deg = __ldg(P.brow + i + 1) - rs;
-                    unsigned long long acc = 0;
+                    W2 acc{0ull, 0ull};
 #pragma unroll
                     for (int k = 0; k < kLight; k++)
-                        if (k < (int)deg) acc |= fr_word(F, bm, __ldg(P.badj + rs + k) & kIdMask);
-                    nw = acc & ~vis;
-                    if (nw) {
-                        P.vis[i] = vis | nw;
-                        Nx[i] = nw;
-                        nowfull = (vis | nw) == full;
-                    } else {
-                        nowfull = vis == full;
+                        if (k < (int)deg) {
+                            const W2 w = fr_word2(F, bm, __ldg(P.badj + rs + k) & kIdMask);
+                            acc.a |= w.a;
+                            acc.b |= w.b;
+                        }
+                    nw = W2{acc.a & ~vis.a, acc.b & ~vis.b};
+                    const W2 nv{vis.a | nw.a, vis.b | nw.b};
+                    if (nw.a | nw.b) {
+                        st2(P.vis + 2 * (size_t)i, nv);
+                        st2(Nx + 2 * (size_t)i, nw);
                     }
+                    nowfull = nv.a == full.a && nv.b == full.b;
                 }
-                const uint32_t fb = __ballot_sync(0xFFFFFFFFu, nw != 0);
+                const uint32_t fb = __ballot_sync(0xFFFFFFFFu, (nw.a | nw.b) != 0);
                 if (fb) {
                     // per-tree discovery counts: transpose the warp's 32 words
-                    // so that lane t counts tree t (and t + 32)
-                    const uint32_t clo = __popc(transpose32((uint32_t)nw));
-                    const uint32_t chi = __popc(transpose32((uint32_t)(nw >> 32)));
-                    if (clo) atomicAdd(&s_cnt[lane], clo);
-                    if (chi) atomicAdd(&s_cnt[lane + 32], chi);
+                    // so that lane t counts trees t, t + 32, t + 64, t + 96
+                    const uint32_t c0 = __popc(transpose32((uint32_t)nw.a));
+                    const uint32_t c1 = __popc(transpose32((uint32_t)(nw.a >> 32)));
+                    if (c0) atomicAdd(&s_cnt[lane], c0);
+                    if (c1) atomicAdd(&s_cnt[lane + 32], c1);
+                    if (__any_sync(0xFFFFFFFFu, nw.b != 0)) {
+                        const uint32_t c2 = __popc(transpose32((uint32_t)nw.b));
+                        const uint32_t c3 = __popc(transpose32((uint32_t)(nw.b >> 32)));
+                        if (c2) atomicAdd(&s_cnt[lane + 64], c2);
+                        if (c3) atomicAdd(&s_cnt[lane + 96], c3);
+                    }
                 }
                 const uint32_t nf = __ballot_sync(0xFFFFFFFFu, nowfull);
                 if (lane == 0 && fb) atomicAdd(&s_fc, (uint32_t)__popc(fb));
@@ -698,22 +745,28 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                     const uint2 it = __ldg(P.items + k);
                     const uint32_t i = it.x;
                     if (!bm_test(nbm, i)) continue;
-                    const unsigned long long nw = __ldcg(Nx + i);
+                    const W2 nw2 = ld2(Nx + 2 * (size_t)i);
                     const uint32_t s1 = min(it.y + (uint32_t)kChunk, __ldg(P.brow + i + 1));
                     const uint32_t ow = __ldg(P.bord + i);
-                    uint32_t p0, p1;
-                    if (s1 - it.y <= 32) {
-                        ms_item_parents(P, F, bm, it.y, s1, nw, ow, s_tk, W, p0, p1);
-                    } else {
-                        unsigned long long b0, b1;
-                        ms_chunk_keys(P, F, bm, it.y, s1, nw, ow, s_tk, true, b0, b1);
-                        p0 = key_to_par(b0);
-                        p1 = key_to_par(b1);
+                    for (int h = 0; h < 2; h++) {
+                        const unsigned long long nw = h ? nw2.b : nw2.a;
+                        if (!nw) continue;   // warp-uniform
+                        const int tb = 64 * h;
+                        uint32_t p0, p1;
+                        if (s1 - it.y <= 32) {
+                            ms_item_parents(P, F, bm, it.y, s1, nw, ow, s_tk + tb, W, p0, p1, h);
+                        } else {
+                            unsigned long long b0, b1;
+                            ms_chunk_keys(P, F, bm, it.y, s1, nw, ow, s_tk + tb, true, b0, b1, h);
+                            p0 = key_to_par(b0);
+                            p1 = key_to_par(b1);
+                        }
+                        if ((nw >> lane) & 1ull)
+                            ms_emit_par(P, tb + lane, s_base[tb + lane] + atomicAdd(&s_pos[tb + lane], 1u), i, p0);
+                        if ((nw >> (lane + 32)) & 1ull)
+                            ms_emit_par(P, tb + lane + 32,
+                                        s_base[tb + lane + 32] + atomicAdd(&s_pos[tb + lane + 32], 1u), i, p1);
                     }
-                    if ((nw >> lane) & 1ull)
-                        ms_emit_par(P, lane, s_base[lane] + atomicAdd(&s_pos[lane], 1u), i, p0);
-                    if ((nw >> (lane + 32)) & 1ull)
-                        ms_emit_par(P, lane + 32, s_base[lane + 32] + atomicAdd(&s_pos[lane + 32], 1u), i, p1);
                 }
             } else {
                 // light vertices: the warp queues its discovered vertices and
@@ -732,12 +785,17 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                     __syncwarp();
                     s_q[wid][lane] = rest;
                     qn -= 32;
-                    ms_light_parents(P, F, Nx, bm, i, true, s_tk, s_base, s_pos, W);
+                    ms_light_parents(P, F, Nx, bm, i, true, s_tk, s_base, s_pos, W, 0);
+                    if (B > 64) ms_light_parents(P, F, Nx, bm, i, true, s_tk + 64, s_base + 64, s_pos + 64, W, 1);
                 }
             }
         }
         __syncwarp();
-        if (qn) ms_light_parents(P, F, Nx, bm, s_q[wid][lane], lane < qn, s_tk, s_base, s_pos, W);
+        if (qn) {
+            ms_light_parents(P, F, Nx, bm, s_q[wid][lane], lane < qn, s_tk, s_base, s_pos, W, 0);
+            if (B > 64)
+                ms_light_parents(P, F, Nx, bm, s_q[wid][lane], lane < qn, s_tk + 64, s_base + 64, s_pos + 64, W, 1);
+        }
         qn = 0;
         // the push bitmap of level L + 1 starts empty
         for (int64_t w = gtid; w < P.nwords; w += nthr) P.tb[(size_t)((L + 1) & 1) * P.nwords + w] = 0;
@@ -747,13 +805,17 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
             for (int64_t k = gwarp; k < P.nmulti_items; k += nwarps) {
                 const uint2 it = __ldg(P.items + k);
                 const uint32_t hi = it.x;
-                const unsigned long long want = __ldcg(P.hacc + hi);
-                if (!want) continue;
+                const W2 want2 = ld2(P.hacc + 2 * (size_t)hi);
+                if (!(want2.a | want2.b)) continue;
                 const uint32_t e1 = min(it.y + (uint32_t)kChunk, __ldg(P.brow + hi + 1));
-                unsigned long long b0, b1;
-                ms_chunk_keys(P, F, bm, it.y, e1, want, __ldg(P.bord + hi), s_tk, false, b0, b1);
-                if (b0 != ~0ull) atomicMin(P.hbest + (size_t)hi * kMsBatch + lane, b0);
-                if (b1 != ~0ull) atomicMin(P.hbest + (size_t)hi * kMsBatch + lane + 32, b1);
+                for (int h = 0; h < 2; h++) {
+                    const unsigned long long want = h ? want2.b : want2.a;
+                    if (!want) continue;
+                    unsigned long long b0, b1;
+                    ms_chunk_keys(P, F, bm, it.y, e1, want, __ldg(P.bord + hi), s_tk + 64 * h, false, b0, b1, h);
+                    if (b0 != ~0ull) atomicMin(P.hbest + (size_t)hi * kMsBatch + 64 * h + lane, b0);
+                    if (b1 != ~0ull) atomicMin(P.hbest + (size_t)hi * kMsBatch + 64 * h + lane + 32, b1);
+                }
             }
         }
         if (blockIdx.x == 0 && tid == 0) P.flag[(L + 1) & 1] = 0;
@@ -762,12 +824,13 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
         // ---------------- phase C: hubs -----------------------------------------
         if (multi) {
             for (int64_t hi = gwarp; hi < P.nmulti; hi += nwarps) {
-                const unsigned long long want = __ldcg(P.hacc + hi);
-                if (!want) continue;
+                const W2 want2 = ld2(P.hacc + 2 * (size_t)hi);
+                if (!(want2.a | want2.b)) continue;
 #pragma unroll
-                for (int h = 0; h < 2; h++) {
-                    const int t = lane + 32 * h;
-                    if ((want >> t) & 1ull) {
+                for (int q = 0; q < 4; q++) {
+                    const int t = lane + 32 * q;
+                    const unsigned long long want = q < 2 ? want2.a : want2.b;
+                    if ((want >> (t & 63)) & 1ull) {
                         unsigned long long *slot = P.hbest + (size_t)hi * kMsBatch + t;
                         const unsigned long long key = __ldcg(slot);
                         *slot = ~0ull;
@@ -779,12 +842,13 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                 __syncwarp();
                 if (lane == 0) {
                     atomicAdd(P.fcnt + (L + 1) % 3, 1u);
-                    const unsigned long long vis = __ldcg(P.vis + hi) | want;
-                    P.vis[hi] = vis;
-                    Nx[hi] = want;
-                    P.hacc[hi] = 0;
+                    const W2 v0 = ld2(P.vis + 2 * (size_t)hi);
+                    const W2 vis{v0.a | want2.a, v0.b | want2.b};
+                    st2(P.vis + 2 * (size_t)hi, vis);
+                    st2(Nx + 2 * (size_t)hi, want2);
+                    st2(P.hacc + 2 * (size_t)hi, W2{0ull, 0ull});
                     atomicOr(nbm + (hi >> 5), 1u << (hi & 31));
-                    if (vis == full) {
+                    if (vis.a == full.a && vis.b == full.b) {
                         atomicOr(P.fullbm + (hi >> 5), 1u << (hi & 31));
                         atomicAdd(P.fcnt + 3, 1u);
                     }
@@ -838,7 +902,8 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
     P.nwords = (g.n + 31) / 32;
     P.itemwords = (g.nlight0 + 31) / 32;
     P.B = B;
-    P.full = B == 64 ? ~0ull : ((1ull << B) - 1);
+    P.full0 = B >= 64 ? ~0ull : ((1ull << B) - 1);
+    P.full1 = B >= 128 ? ~0ull : B > 64 ? ((1ull << (B - 64)) - 1) : 0ull;
     P.vis = ws.vis; P.fr = ws.fr; P.hacc = ws.hacc; P.hbest = ws.hbest;
     P.fbm = ws.fbm; P.fullbm = ws.fbm + 3 * P.nwords;
     P.tb = ws.fbm + 4 * P.nwords;
@@ -848,8 +913,8 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
     P.tkey = o.tkey; P.qv = o.qv; P.parq = o.parq; P.pp = o.pp; P.rec = o.rec; P.crec = o.crec; P.irec = o.irec;
     P.lvl = o.lvl; P.vbase = o.vbase; P.depth = o.depth; P.maxd = o.maxd;
     P.prof = ws.msprof;
-    GB_CUDA_TRY(cudaMemsetAsync(ws.vis, 0, sizeof(unsigned long long) * (size_t)g.n, st));
-    GB_CUDA_TRY(cudaMemsetAsync(ws.fr, 0, sizeof(unsigned long long) * (size_t)g.n, st));
+    GB_CUDA_TRY(cudaMemsetAsync(ws.vis, 0, sizeof(unsigned long long) * 2 * (size_t)g.n, st));
+    GB_CUDA_TRY(cudaMemsetAsync(ws.fr, 0, sizeof(unsigned long long) * 2 * (size_t)g.n, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.fbm, 0, sizeof(uint32_t) * 6 * (size_t)P.nwords, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.msflag, 0, sizeof(int32_t) * 8, st));
     const int64_t work = std::max<int64_t>((int64_t)B * g.nbig, g.niso);

@@ -24,6 +24,7 @@ def _free_port():
 
 
 def _worker(rank, world, port, T, seed, out):
+    from datetime import timedelta
     import torch
     import torch.distributed as dist
     os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -31,11 +32,12 @@ def _worker(rank, world, port, T, seed, out):
     ndev = torch.cuda.device_count()
     torch.cuda.set_device(rank % ndev)
     backend = "nccl" if ndev >= world else "gloo"
+    # a rank that dies must not leave the other waiting forever
     if backend == "nccl":
-        dist.init_process_group("nccl", rank=rank, world_size=world,
+        dist.init_process_group("nccl", rank=rank, world_size=world, timeout=timedelta(seconds=300),
                                 device_id=torch.device("cuda", rank % ndev))
     else:
-        dist.init_process_group("gloo", rank=rank, world_size=world)
+        dist.init_process_group("gloo", rank=rank, world_size=world, timeout=timedelta(seconds=300))
     try:
         import graphgen
         from paper_conf_sc_alabanditrb21_b200 import graphb

@@ -109,6 +109,16 @@ def test_power_law_hubs_multi_batch(walk, linear):
     check_cloud(g, 37, 11, batch=16, cycle_group=5, walk=walk, desc_linear=linear)
 
 
+def test_msbfs_128_tree_pass():
+    """One multi-source BFS pass holds up to 128 trees (two 64-bit halves per
+    vertex): 130 trees = a 128-tree batch + a 2-tree batch on a graph with
+    hubs (multi-chunk vertices, phase C) and isolated vertices; the whole
+    cloud and every per-tree statistic against the oracle."""
+    g = graphgen.chung_lu(6000, 30000, 1500, 0.75, 0.3, 21, lcc=False)
+    st = check_cloud(g, 130, 4)
+    assert st["batch"] == 128 and st["batches"] == 2
+
+
 @pytest.mark.parametrize("walk", [1, 2])
 def test_paper_walks_on_forests_and_degenerate_trees(walk):
     """Walks 1 and 2 on a forest with isolated vertices (roots without a
@@ -391,23 +401,23 @@ def test_c4_epinions_tree_subset():
 @pytest.mark.slow
 def test_c3_amazon_sampled_trees():
     """C3 (10M / 22M) at full size in bench's launch configuration (one step:
-    100 trees as MS-BFS batches of 64 + 36, one tree per labelling launch):
+    100 trees in one 128-wide MS-BFS pass, four trees per labelling launch):
     per-tree statistics of all trees against invariants, and four sampled
     trees (first / last of each batch) bit-exact against the oracle -- cycle
     lengths, depth and the signature of the switched edge set."""
     g, T, _ = graphgen.config("c3")
     assert T == 100
     graphb.load_graph(g)
-    cnt, agree = graphb.balance_host(T, 1)      # bench's step: batches of 64 + 36 trees
+    cnt, agree = graphb.balance_host(T, 1)      # bench's step: one batch of 100 trees
     st = graphb.stats()
-    assert st["batch"] == 64 and st["batches"] == 2
+    assert st["batch"] == 100 and st["batches"] == 1 and st["sub"] == 4
     ids, per = graphb.tree_stats()
     og = oracle.Graph.from_csr(g)
     c = og.ncomp
     assert np.all(per[:, 1] == g.m - g.n + c)                  # L112
     assert np.all(agree <= 2 * T) and cnt.max() <= T
-    # sampled trees of both batches (first / last of each): cycle lengths,
-    # depth and the signature of the switched edge set, bit-exact
+    # sampled trees of both 64-tree halves of the pass (first / last of
+    # each): cycle lengths, depth and the signature of the switched edge set
     for t in (0, 63, 64, 99):
         parent, dist, _ = og.bfs_tree(1, t)
         flip, sk, nc, md = og.balance_tree(parent)
