@@ -50,6 +50,7 @@ struct Options {
     int64_t cycle_group = 0; // 0 = auto
     int64_t walk = 0;        // 0 two-ended, 1 Alg. 3 descent (child lists), 2 the paper's edge lists (L238-L244)
     int64_t desc_linear = 0; // walk 1: 1 = linear int4 ballot rounds over the child starts, 0 = 32-ary pivots
+    int64_t walk_ept = 1;    // walk 0 (layout 0): edges per thread, climbed interleaved (1, 2, 4)
     int64_t timing = 0;
     int64_t sub = 0;         // trees per labelling launch (0 = auto)
     int64_t msprof = 0;      // record BFS phase timestamps (gb_msbfs_profile)
@@ -451,7 +452,8 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
                             bfs_opts());
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
-        rc = run_batch_cycles(S.g, S.ws, nb, G, (int)S.opt.walk, st, &T.launches, jump, (int)S.opt.desc_linear);
+        rc = run_batch_cycles(S.g, S.ws, nb, G, (int)S.opt.walk, st, &T.launches, jump, (int)S.opt.desc_linear,
+                              (int)S.opt.walk_ept);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[5], st));
         if (S.opt.harary) {
@@ -516,7 +518,8 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
             return GB_EINVAL;
         }
     }
-    rc = run_batch_cycles(S.g, S.ws, 1, 1, (int)S.opt.walk, st, &T.launches, 1, (int)S.opt.desc_linear);
+    rc = run_batch_cycles(S.g, S.ws, 1, 1, (int)S.opt.walk, st, &T.launches, 1, (int)S.opt.desc_linear,
+                          (int)S.opt.walk_ept);
     if (rc) return rc;
     GB_CUDA_TRY(cudaStreamSynchronize(st));
     return GB_OK;
@@ -673,6 +676,10 @@ int gb_set_option(const char *key, int64_t value) {
         S.opt.walk = value;
     }
     else if (!strcmp(key, "desc_linear")) S.opt.desc_linear = value != 0;
+    else if (!strcmp(key, "walk_ept")) {
+        if (value != 1 && value != 2 && value != 4) { set_error("walk_ept must be 1, 2 or 4"); return GB_EINVAL; }
+        S.opt.walk_ept = value;
+    }
     else if (!strcmp(key, "timing")) S.opt.timing = value != 0;
     else if (!strcmp(key, "sub")) { if (value < 0) return GB_EINVAL; S.opt.sub = value; }
     else if (!strcmp(key, "msprof")) S.opt.msprof = value != 0;

@@ -206,6 +206,87 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_irec(CycleParams P) {
     flush_stats(P, s_k, s_c, s_sig);
 }
 
+// The same walk with EPT edges per thread (EPT consecutive 32-edge words per
+// warp), their climbs interleaved: 2 * EPT independent gathers in flight per
+// thread, and a lane idles only once all its edges are done (the cycle
+// lengths of one edge vary a lot; the sum over EPT edges less so).
+template <int EPT>
+__global__ void __launch_bounds__(kCycleBlock) k_cycles_irec_m(CycleParams P) {
+    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup], s_sig[kMaxGroup];
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; s_sig[i] = 0; }
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t w0 = gw * EPT; w0 < P.words; w0 += nw * EPT) {
+        uint32_t u[EPT], v[EPT], nege[EPT];
+        bool valid[EPT];
+#pragma unroll
+        for (int j = 0; j < EPT; j++) {
+            const int64_t e = (w0 + j) * 32 + lane;
+            valid[j] = w0 + j < P.words && e < P.m;
+            const uint2 ed = valid[j] ? __ldg(P.edges + e) : make_uint2(0, 0);
+            u[j] = ed.x;
+            v[j] = ed.y & kIdMask;
+            nege[j] = ed.y >> 31;
+        }
+        for (int g = 0; g < P.G; g++) {
+            const uint4 *rec = P.irec + (size_t)(P.b0 + g) * P.n;
+            uint4 rx[EPT], ry[EPT];
+            uint32_t px[EPT], py[EPT], c[EPT], k[EPT];
+            bool ax[EPT], ay[EPT], cyc[EPT];
+#pragma unroll
+            for (int j = 0; j < EPT; j++) {
+                rx[j] = valid[j] ? __ldg(rec + u[j]) : make_uint4(0, 0, 1, 0);
+                ry[j] = valid[j] ? __ldg(rec + v[j]) : make_uint4(0, 0, 1, 0);
+            }
+#pragma unroll
+            for (int j = 0; j < EPT; j++) {
+                // tree edge iff one endpoint is the other's parent (simple graph)
+                cyc[j] = valid[j] && (rx[j].x & kIdMask) != v[j] && (ry[j].x & kIdMask) != u[j];
+                px[j] = rx[j].y & kIdMask;
+                py[j] = ry[j].y & kIdMask;
+                c[j] = 0;
+                k[j] = cyc[j] ? 1u : 0u;
+                ax[j] = !cyc[j] || is_anc(px[j], rx[j].z, py[j]);
+                ay[j] = !cyc[j] || is_anc(py[j], ry[j].z, px[j]);
+            }
+            for (;;) {
+                bool more = false;
+#pragma unroll
+                for (int j = 0; j < EPT; j++) {
+                    if (!ax[j]) {
+                        c[j] ^= rx[j].x;
+                        rx[j] = __ldg(rec + (rx[j].x & kIdMask));
+                        k[j]++;
+                    }
+                    if (!ay[j]) {
+                        c[j] ^= ry[j].x;
+                        ry[j] = __ldg(rec + (ry[j].x & kIdMask));
+                        k[j]++;
+                    }
+                }
+#pragma unroll
+                for (int j = 0; j < EPT; j++) {
+                    if (!ax[j]) ax[j] = is_anc(rx[j].y & kIdMask, rx[j].z, py[j]);
+                    if (!ay[j]) ay[j] = is_anc(ry[j].y & kIdMask, ry[j].z, px[j]);
+                    more |= !(ax[j] && ay[j]);
+                }
+                if (!more) break;
+            }
+#pragma unroll
+            for (int j = 0; j < EPT; j++) {
+                const uint32_t flip = cyc[j] ? (c[j] >> 31) ^ nege[j] : 0u;
+                const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
+                if (lane == 0 && w0 + j < P.words) P.fbits[(size_t)(P.b0 + g) * P.words + w0 + j] = bits;
+                warp_stats(lane, g, k[j], cyc[j], flip != 0, (w0 + j) * 32 + lane, s_k, s_c, s_sig);
+            }
+        }
+    }
+    __syncthreads();
+    flush_stats(P, s_k, s_c, s_sig);
+}
+
 // ---------------------------------------------------------------------------
 // K-level records for the two-ended walk (option "jump"): jrec[x][j] =
 // rec[a_j(x)], a_0 = x, a_{j+1} = parent of a_j (the root is its own parent).
@@ -580,7 +661,7 @@ static unsigned grid_cap(int64_t work, int threads, int sms, int per_sm) {
 }
 
 int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, int walk,
-                     cudaStream_t st, int64_t *launches, int jump, int linear) {
+                     cudaStream_t st, int64_t *launches, int jump, int linear, int ept) {
     CycleParams P;
     const bool descent = walk == 1, paper = walk == 2;
     if (walk != 0 || !ws.jrec) jump = 1;
@@ -625,6 +706,8 @@ int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, int walk,
             P.tbase = ws.ptbase; P.tnbr = ws.ptnbr; P.trng = ws.ptrng;
             k_cycles_paper<<<grid, kCycleBlock, 0, st>>>(P);
         }
+        else if (irec && ept == 2) k_cycles_irec_m<2><<<grid_cap(P.words * 16, kCycleBlock, g.num_sms, 8), kCycleBlock, 0, st>>>(P);
+        else if (irec && ept == 4) k_cycles_irec_m<4><<<grid_cap(P.words * 8, kCycleBlock, g.num_sms, 8), kCycleBlock, 0, st>>>(P);
         else if (irec) k_cycles_irec<<<grid, kCycleBlock, 0, st>>>(P);
         else if (descent) k_cycles_descent<<<grid, kCycleBlock, 0, st>>>(P);
         else if (jump == 2) k_cycles_jump<2><<<grid, kCycleBlock, 0, st>>>(P);

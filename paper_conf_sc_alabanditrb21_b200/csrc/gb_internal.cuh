@@ -306,7 +306,7 @@ int debug_tree_views(const Graph &g, Workspace &ws, bool descent, int32_t *d_par
 // walk: 0 two-ended, 1 Alg. 3 descent over child lists, 2 the paper's
 // partitioned two-word edge lists (linear scan)
 int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, int walk,
-                     cudaStream_t st, int64_t *launches, int jump = 1, int linear = 0);
+                     cudaStream_t st, int64_t *launches, int jump = 1, int linear = 0, int ept = 1);
 
 int run_batch_accumulate(const Graph &g, Workspace &ws, int B, int32_t *d_cnt,
                          int32_t *d_agree, cudaStream_t st, int64_t *launches);

@@ -481,6 +481,19 @@ __global__ void k_ms_roots(MsParams P) {
             }
         }
     }
+    // ... and finished from the start: their "finished" bits are set (the
+    // discovery passes skip them) and counted once
+    if (P.niso > 0) {
+        const int64_t i0 = P.n - P.niso;
+        for (int64_t w = (i0 >> 5) + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < P.nwords;
+             w += (int64_t)gridDim.x * blockDim.x) {
+            uint32_t m = ~0u;
+            if ((w << 5) < i0) m &= ~0u << (uint32_t)(i0 - (w << 5));
+            if (((w + 1) << 5) > P.n) m &= ~0u >> (uint32_t)(((w + 1) << 5) - P.n);
+            atomicOr(P.fullbm + w, m);
+        }
+        if (blockIdx.x == 0 && threadIdx.x == 0) P.fcnt[3] = (uint32_t)P.niso;
+    }
     const int64_t total = (int64_t)P.B * P.nbig;
     for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < total;
          x += (int64_t)gridDim.x * blockDim.x) {
@@ -571,7 +584,8 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
         // neighbours in tbc -- so that the pull below reads the adjacency of
         // marked vertices only (nothing else can be discovered).  Heavy
         // vertices push through their work items (<= 256 slots per warp).
-        const uint32_t fc = L == 0 ? (uint32_t)(((int64_t)B * P.ncomp < P.n) ? (int64_t)B * P.ncomp : P.n)
+        // level 0: one root per tree in every component with >= 2 vertices
+        const uint32_t fc = L == 0 ? (uint32_t)(((int64_t)B * P.nbig < P.n) ? (int64_t)B * P.nbig : P.n)
                                    : __ldcg(P.fcnt + L % 3);
         const int64_t unfinished = P.n - (int64_t)__ldcg(P.fcnt + 3);
         const bool push = (int64_t)fc * P.push_div <= unfinished;

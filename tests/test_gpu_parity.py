@@ -109,6 +109,15 @@ def test_power_law_hubs_multi_batch(walk, linear):
     check_cloud(g, 37, 11, batch=16, cycle_group=5, walk=walk, desc_linear=linear)
 
 
+@pytest.mark.parametrize("ept", [2, 4])
+def test_walk_edges_per_thread(ept):
+    """Walk 0 with 2 / 4 edges per thread climbed interleaved (option
+    walk_ept), cycle groups and a ragged last word (m not a multiple of 32)."""
+    g = graphgen.chung_lu(20000, 90001, 2500, 0.75, 0.25, 3)
+    check_cloud(g, 37, 11, batch=16, cycle_group=5, walk_ept=ept)
+    check_cloud(graphgen.er(5000, 3000, 0.4, 2), 9, 3, walk_ept=ept)
+
+
 def test_msbfs_128_tree_pass():
     """One multi-source BFS pass holds up to 128 trees (two 64-bit halves per
     vertex): 130 trees = a 128-tree batch + a 2-tree batch on a graph with
