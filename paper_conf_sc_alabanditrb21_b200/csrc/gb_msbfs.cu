@@ -104,25 +104,39 @@ __device__ __forceinline__ bool bm_test(const uint32_t *bm, uint32_t u) {
 struct W2 {
     unsigned long long a, b;   // trees 0-63, 64-127
 };
+// S = words per vertex: 2 (batches of 65..128 trees, interleaved halves) or 1
+// (<= 64 trees: the round-1 layout, 8-byte loads)
+template <int S>
 __device__ __forceinline__ W2 ld2(const unsigned long long *p) {
-    const uint4 v = __ldcg(reinterpret_cast<const uint4 *>(p));
-    return W2{(unsigned long long)v.x | ((unsigned long long)v.y << 32),
-              (unsigned long long)v.z | ((unsigned long long)v.w << 32)};
+    if constexpr (S == 1) {
+        return W2{__ldcg(p), 0ull};
+    } else {
+        const uint4 v = __ldcg(reinterpret_cast<const uint4 *>(p));
+        return W2{(unsigned long long)v.x | ((unsigned long long)v.y << 32),
+                  (unsigned long long)v.z | ((unsigned long long)v.w << 32)};
+    }
 }
+template <int S>
 __device__ __forceinline__ void st2(unsigned long long *p, W2 w) {
-    *reinterpret_cast<uint4 *>(p) = make_uint4((uint32_t)w.a, (uint32_t)(w.a >> 32), (uint32_t)w.b,
-                                               (uint32_t)(w.b >> 32));
+    if constexpr (S == 1) {
+        *p = w.a;
+    } else {
+        *reinterpret_cast<uint4 *>(p) = make_uint4((uint32_t)w.a, (uint32_t)(w.a >> 32), (uint32_t)w.b,
+                                                   (uint32_t)(w.b >> 32));
+    }
 }
 
 // half h of the frontier word of u (0 unless u is on the current level in
 // some tree)
+template <int S>
 __device__ __forceinline__ unsigned long long fr_word(const unsigned long long *F, const uint32_t *bm,
                                                       uint32_t u, int h) {
-    return bm_test(bm, u) ? __ldcg(F + 2 * (size_t)u + h) : 0ull;
+    return bm_test(bm, u) ? __ldcg(F + S * (size_t)u + h) : 0ull;
 }
-// both halves (one 16-byte load)
+// both halves (one 16-byte load when S = 2)
+template <int S>
 __device__ __forceinline__ W2 fr_word2(const unsigned long long *F, const uint32_t *bm, uint32_t u) {
-    return bm_test(bm, u) ? ld2(F + 2 * (size_t)u) : W2{0ull, 0ull};
+    return bm_test(bm, u) ? ld2<S>(F + S * (size_t)u) : W2{0ull, 0ull};
 }
 
 // level-(L+1) entry `pos` of tree t: the vertex and its parent | neg << 31,
@@ -144,6 +158,7 @@ __device__ __forceinline__ void ms_emit_par(const MsParams &P, int t, uint32_t p
 }
 
 // OR of the frontier words over the slots [s0, s1) (one warp, lanes stride)
+template <int S>
 __device__ __forceinline__ W2 ms_chunk_or(const MsParams &P, const unsigned long long *F,
                                           const uint32_t *bm, uint32_t s0, uint32_t s1) {
     const int lane = threadIdx.x & 31;
@@ -152,13 +167,13 @@ __device__ __forceinline__ W2 ms_chunk_or(const MsParams &P, const unsigned long
     for (; j + 96 < s1; j += 128) {
         const uint32_t a0 = __ldg(P.badj + j) & kIdMask, a1 = __ldg(P.badj + j + 32) & kIdMask;
         const uint32_t a2 = __ldg(P.badj + j + 64) & kIdMask, a3 = __ldg(P.badj + j + 96) & kIdMask;
-        const W2 w0 = fr_word2(F, bm, a0), w1 = fr_word2(F, bm, a1);
-        const W2 w2 = fr_word2(F, bm, a2), w3 = fr_word2(F, bm, a3);
+        const W2 w0 = fr_word2<S>(F, bm, a0), w1 = fr_word2<S>(F, bm, a1);
+        const W2 w2 = fr_word2<S>(F, bm, a2), w3 = fr_word2<S>(F, bm, a3);
         acc.a |= w0.a | w1.a | w2.a | w3.a;
         acc.b |= w0.b | w1.b | w2.b | w3.b;
     }
     for (; j < s1; j += 32) {
-        const W2 w = fr_word2(F, bm, __ldg(P.badj + j) & kIdMask);
+        const W2 w = fr_word2<S>(F, bm, __ldg(P.badj + j) & kIdMask);
         acc.a |= w.a;
         acc.b |= w.b;
     }
@@ -178,6 +193,7 @@ __device__ __forceinline__ unsigned long long warp_min64(unsigned long long v) {
 // chunk is the whole adjacency and fits one window, a tree with a single
 // candidate takes it without hashing (its key then has score 0, which only
 // matters for the decode).
+template <int S>
 __device__ __forceinline__ void ms_chunk_keys(const MsParams &P, const unsigned long long *F,
                                               const uint32_t *bm, uint32_t s0, uint32_t s1,
                                               unsigned long long want, uint32_t ow, const uint64_t *s_tk,
@@ -193,7 +209,7 @@ __device__ __forceinline__ void ms_chunk_keys(const MsParams &P, const unsigned 
         unsigned long long f = 0;
         if (j < s1) {
             const uint32_t a = __ldg(P.badj + j);
-            f = fr_word(F, bm, a & kIdMask, h) & want;
+            f = fr_word<S>(F, bm, a & kIdMask, h) & want;
             if (f) o = __ldg(P.borig + j) | (a & kNegBit);
         }
         for (unsigned long long rem = warp_or64(f); rem; rem &= rem - 1) {
@@ -260,6 +276,7 @@ __device__ __forceinline__ uint32_t transpose32(uint32_t x) {
 // tree's level list with one shared-memory add and writes its entries.
 // Half h of the 128 trees (trees 64h .. 64h + 63; s_tk, s_base and s_pos
 // point at the half's first tree).
+template <int S>
 __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsigned long long *F,
                                                  const unsigned long long *Nx, const uint32_t *bm,
                                                  uint32_t i, bool act, const uint64_t *s_tk,
@@ -269,7 +286,7 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
     unsigned long long nw = 0, s2m = 0;   // discovered trees / those with >= 2 candidates
     unsigned long long c[kLight];
     uint32_t ow = 0;
-    if (act) nw = __ldcg(Nx + 2 * (size_t)i + half);
+    if (act) nw = __ldcg(Nx + S * (size_t)i + half);
     if (!__any_sync(0xFFFFFFFFu, nw != 0)) return;   // nothing in this half
     if (act) {
         const uint32_t rs = __ldg(P.brow + i);
@@ -281,7 +298,7 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
             c[k] = 0;
             if (k < (int)deg) {
                 const uint32_t a = __ldg(P.badj + rs + k);
-                c[k] = fr_word(F, bm, a & kIdMask, half) & nw;
+                c[k] = fr_word<S>(F, bm, a & kIdMask, half) & nw;
                 if (c[k]) {
                     W.lo[k][lane] = __ldg(P.borig + rs + k) | (a & kNegBit);
                     W.li[k][lane] = a;
@@ -387,6 +404,7 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
 // <= 32; lane = slot) in the trees `want`: trees with one candidate take it,
 // the (slot, tree) pairs of the others are hashed one per lane and reduced
 // with shared-memory atomicMin.  Lanes l, l + 32 get trees l, l + 32.
+template <int S>
 __device__ __forceinline__ void ms_item_parents(const MsParams &P, const unsigned long long *F,
                                                 const uint32_t *bm, uint32_t s0, uint32_t s1,
                                                 unsigned long long want, uint32_t ow,
@@ -399,7 +417,7 @@ __device__ __forceinline__ void ms_item_parents(const MsParams &P, const unsigne
     uint32_t o = 0;
     if (j < s1) {
         const uint32_t a = __ldg(P.badj + j);
-        f = fr_word(F, bm, a & kIdMask, h) & want;
+        f = fr_word<S>(F, bm, a & kIdMask, h) & want;
         if (f) o = __ldg(P.borig + j) | (a & kNegBit);
     }
     unsigned long long s1m = f, s2m = 0;   // trees with >= 1 / >= 2 candidates
@@ -461,6 +479,7 @@ __device__ __forceinline__ int select_bit64(unsigned long long m, int r) {
 // roots (reading R4): root of component C in tree b = C's vertices
 // (ascending)[rkey(b, C) mod |C|]; level 0 of every tree
 // ---------------------------------------------------------------------------
+template <int S>
 __global__ void k_ms_roots(MsParams P) {
     // single-vertex components (the isolated vertices, internal ids
     // [n - niso, n)): their one-vertex trees are identical in every tree --
@@ -468,7 +487,7 @@ __global__ void k_ms_roots(MsParams P) {
     // coff[C], pi = 0, size 1 (read from the component table wherever needed)
     for (int64_t i = P.n - P.niso + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.n;
          i += (int64_t)gridDim.x * blockDim.x) {
-        st2(P.vis + 2 * i, W2{P.full0, P.full1});
+        st2<S>(P.vis + S * i, W2{P.full0, P.full1});
         if (!P.irec) {
             // layout 1 (walks 1, 2, option jump) reads pre-indexed records of
             // every vertex: the one-vertex trees' records, per tree
@@ -505,13 +524,13 @@ __global__ void k_ms_roots(MsParams P) {
         const uint32_t ri = P.brank[r];
         const unsigned long long bit = 1ull << (b & 63);
         const int h = b >> 6;
-        atomicOr(P.vis + 2 * (size_t)ri + h, bit);
+        atomicOr(P.vis + S * (size_t)ri + h, bit);
         const size_t nb = (size_t)b * P.n;
         const unsigned long long old = atomicAdd((unsigned long long *)(P.lvl + b * P.ls), 1ull << 32);
         const uint32_t pos = (uint32_t)(old >> 32);
         P.qv[nb + pos] = ri;
         P.parq[nb + pos] = ri;
-        atomicOr(P.fr + 2 * (size_t)ri + h, bit);
+        atomicOr(P.fr + S * (size_t)ri + h, bit);
         atomicOr(P.fbm + (ri >> 5), 1u << (ri & 31));
     }
 }
@@ -530,6 +549,7 @@ __global__ void k_ms_roots(MsParams P) {
 //   phase C  (only if a hub discovered something) hubs' parents appended,
 //            then one more barrier.
 // ---------------------------------------------------------------------------
+template <int S>
 __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
     cg::grid_group grid = cg::this_grid();
     __shared__ uint64_t s_tk[kMsBatch];
@@ -563,8 +583,8 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
     const uint32_t nblk = gridDim.x;
     __shared__ uint32_t s_fc, s_ff;
     for (int L = 0;; L++) {
-        const unsigned long long *F = P.fr + (size_t)(L & 1) * 2 * P.n;
-        unsigned long long *Nx = P.fr + (size_t)((L + 1) & 1) * 2 * P.n;
+        const unsigned long long *F = P.fr + (size_t)(L & 1) * S * P.n;
+        unsigned long long *Nx = P.fr + (size_t)((L + 1) & 1) * S * P.n;
         const uint32_t *bm = P.fbm + (size_t)(L % 3) * P.nwords;
         uint32_t *nbm = P.fbm + (size_t)((L + 1) % 3) * P.nwords;
         uint32_t *cbm = P.fbm + (size_t)((L + 2) % 3) * P.nwords;   // free: cleared for L+2
@@ -625,21 +645,21 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                     if (push && !bm_test(tbc, i)) continue;
                     const uint32_t s1 = min(s0 + (uint32_t)kChunk, __ldg(P.brow + i + 1));
                     const bool multi = k < P.nmulti_items;
-                    const W2 vis = ld2(P.vis + 2 * (size_t)i);
-                    W2 part = ms_chunk_or(P, F, bm, s0, s1);
+                    const W2 vis = ld2<S>(P.vis + S * (size_t)i);
+                    W2 part = ms_chunk_or<S>(P, F, bm, s0, s1);
                     part.a &= ~vis.a;
                     part.b &= ~vis.b;
                     if (multi) {
                         if ((part.a | part.b) && lane == 0) {
-                            if (part.a) atomicOr(P.hacc + 2 * (size_t)i, part.a);
-                            if (part.b) atomicOr(P.hacc + 2 * (size_t)i + 1, part.b);
+                            if (part.a) atomicOr(P.hacc + S * (size_t)i, part.a);
+                            if (part.b) atomicOr(P.hacc + S * (size_t)i + 1, part.b);
                             P.flag[L & 1] = 1;
                         }
                     } else if (part.a | part.b) {
                         if (lane == 0) {
-                            st2(Nx + 2 * (size_t)i, part);
+                            st2<S>(Nx + S * (size_t)i, part);
                             const W2 nv{vis.a | part.a, vis.b | part.b};
-                            st2(P.vis + 2 * (size_t)i, nv);
+                            st2<S>(P.vis + S * (size_t)i, nv);
                             atomicOr(nbm + (i >> 5), 1u << (i & 31));
                             if (nv.a == full.a && nv.b == full.b) {
                                 atomicOr(P.fullbm + (i >> 5), 1u << (i & 31));
@@ -663,22 +683,22 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                 W2 nw{0ull, 0ull};
                 bool nowfull = false;
                 if (mine && !((fw >> lane) & 1u) && ((tw >> lane) & 1u)) {
-                    const W2 vis = ld2(P.vis + 2 * (size_t)i);
+                    const W2 vis = ld2<S>(P.vis + S * (size_t)i);
                     const uint32_t rs = __ldg(P.brow + i);
                     const uint32_t deg = __ldg(P.brow + i + 1) - rs;
                     W2 acc{0ull, 0ull};
 #pragma unroll
                     for (int k = 0; k < kLight; k++)
                         if (k < (int)deg) {
-                            const W2 w = fr_word2(F, bm, __ldg(P.badj + rs + k) & kIdMask);
+                            const W2 w = fr_word2<S>(F, bm, __ldg(P.badj + rs + k) & kIdMask);
                             acc.a |= w.a;
                             acc.b |= w.b;
                         }
                     nw = W2{acc.a & ~vis.a, acc.b & ~vis.b};
                     const W2 nv{vis.a | nw.a, vis.b | nw.b};
                     if (nw.a | nw.b) {
-                        st2(P.vis + 2 * (size_t)i, nv);
-                        st2(Nx + 2 * (size_t)i, nw);
+                        st2<S>(P.vis + S * (size_t)i, nv);
+                        st2<S>(Nx + S * (size_t)i, nw);
                     }
                     nowfull = nv.a == full.a && nv.b == full.b;
                 }
@@ -759,7 +779,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                     const uint2 it = __ldg(P.items + k);
                     const uint32_t i = it.x;
                     if (!bm_test(nbm, i)) continue;
-                    const W2 nw2 = ld2(Nx + 2 * (size_t)i);
+                    const W2 nw2 = ld2<S>(Nx + S * (size_t)i);
                     const uint32_t s1 = min(it.y + (uint32_t)kChunk, __ldg(P.brow + i + 1));
                     const uint32_t ow = __ldg(P.bord + i);
                     for (int h = 0; h < 2; h++) {
@@ -768,10 +788,10 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                         const int tb = 64 * h;
                         uint32_t p0, p1;
                         if (s1 - it.y <= 32) {
-                            ms_item_parents(P, F, bm, it.y, s1, nw, ow, s_tk + tb, W, p0, p1, h);
+                            ms_item_parents<S>(P, F, bm, it.y, s1, nw, ow, s_tk + tb, W, p0, p1, h);
                         } else {
                             unsigned long long b0, b1;
-                            ms_chunk_keys(P, F, bm, it.y, s1, nw, ow, s_tk + tb, true, b0, b1, h);
+                            ms_chunk_keys<S>(P, F, bm, it.y, s1, nw, ow, s_tk + tb, true, b0, b1, h);
                             p0 = key_to_par(b0);
                             p1 = key_to_par(b1);
                         }
@@ -799,16 +819,16 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                     __syncwarp();
                     s_q[wid][lane] = rest;
                     qn -= 32;
-                    ms_light_parents(P, F, Nx, bm, i, true, s_tk, s_base, s_pos, W, 0);
-                    if (B > 64) ms_light_parents(P, F, Nx, bm, i, true, s_tk + 64, s_base + 64, s_pos + 64, W, 1);
+                    ms_light_parents<S>(P, F, Nx, bm, i, true, s_tk, s_base, s_pos, W, 0);
+                    if (B > 64) ms_light_parents<S>(P, F, Nx, bm, i, true, s_tk + 64, s_base + 64, s_pos + 64, W, 1);
                 }
             }
         }
         __syncwarp();
         if (qn) {
-            ms_light_parents(P, F, Nx, bm, s_q[wid][lane], lane < qn, s_tk, s_base, s_pos, W, 0);
+            ms_light_parents<S>(P, F, Nx, bm, s_q[wid][lane], lane < qn, s_tk, s_base, s_pos, W, 0);
             if (B > 64)
-                ms_light_parents(P, F, Nx, bm, s_q[wid][lane], lane < qn, s_tk + 64, s_base + 64, s_pos + 64, W, 1);
+                ms_light_parents<S>(P, F, Nx, bm, s_q[wid][lane], lane < qn, s_tk + 64, s_base + 64, s_pos + 64, W, 1);
         }
         qn = 0;
         // the push bitmap of level L + 1 starts empty
@@ -819,14 +839,14 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
             for (int64_t k = gwarp; k < P.nmulti_items; k += nwarps) {
                 const uint2 it = __ldg(P.items + k);
                 const uint32_t hi = it.x;
-                const W2 want2 = ld2(P.hacc + 2 * (size_t)hi);
+                const W2 want2 = ld2<S>(P.hacc + S * (size_t)hi);
                 if (!(want2.a | want2.b)) continue;
                 const uint32_t e1 = min(it.y + (uint32_t)kChunk, __ldg(P.brow + hi + 1));
                 for (int h = 0; h < 2; h++) {
                     const unsigned long long want = h ? want2.b : want2.a;
                     if (!want) continue;
                     unsigned long long b0, b1;
-                    ms_chunk_keys(P, F, bm, it.y, e1, want, __ldg(P.bord + hi), s_tk + 64 * h, false, b0, b1, h);
+                    ms_chunk_keys<S>(P, F, bm, it.y, e1, want, __ldg(P.bord + hi), s_tk + 64 * h, false, b0, b1, h);
                     if (b0 != ~0ull) atomicMin(P.hbest + (size_t)hi * kMsBatch + 64 * h + lane, b0);
                     if (b1 != ~0ull) atomicMin(P.hbest + (size_t)hi * kMsBatch + 64 * h + lane + 32, b1);
                 }
@@ -838,7 +858,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
         // ---------------- phase C: hubs -----------------------------------------
         if (multi) {
             for (int64_t hi = gwarp; hi < P.nmulti; hi += nwarps) {
-                const W2 want2 = ld2(P.hacc + 2 * (size_t)hi);
+                const W2 want2 = ld2<S>(P.hacc + S * (size_t)hi);
                 if (!(want2.a | want2.b)) continue;
 #pragma unroll
                 for (int q = 0; q < 4; q++) {
@@ -856,11 +876,11 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                 __syncwarp();
                 if (lane == 0) {
                     atomicAdd(P.fcnt + (L + 1) % 3, 1u);
-                    const W2 v0 = ld2(P.vis + 2 * (size_t)hi);
+                    const W2 v0 = ld2<S>(P.vis + S * (size_t)hi);
                     const W2 vis{v0.a | want2.a, v0.b | want2.b};
-                    st2(P.vis + 2 * (size_t)hi, vis);
-                    st2(Nx + 2 * (size_t)hi, want2);
-                    st2(P.hacc + 2 * (size_t)hi, W2{0ull, 0ull});
+                    st2<S>(P.vis + S * (size_t)hi, vis);
+                    st2<S>(Nx + S * (size_t)hi, want2);
+                    st2<S>(P.hacc + S * (size_t)hi, W2{0ull, 0ull});
                     atomicOr(nbm + (hi >> 5), 1u << (hi & 31));
                     if (vis.a == full.a && vis.b == full.b) {
                         atomicOr(P.fullbm + (hi >> 5), 1u << (hi & 31));
@@ -898,14 +918,19 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
               int64_t *launches) {
     if (B < 1 || B > kMsBatch) { set_error("msbfs: batch out of range"); return GB_EINVAL; }
     // co-resident grid size, recomputed when the device changes (SM count)
-    static int blocks = 0, blocks_dev = -1;
+    const int S = B > 64 ? 2 : 1;   // words per vertex
+    const void *kern = S == 2 ? (const void *)k_msbfs<2> : (const void *)k_msbfs<1>;
+    static int blocks[2] = {0, 0}, blocks_dev = -1;
     if (blocks_dev != g.dev) {
         blocks_dev = g.dev;
-        int per = 0;
-        GB_CUDA_TRY(cudaFuncSetAttribute(k_msbfs, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMsSmem));
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_msbfs, kBlock, kMsSmem) != cudaSuccess || per < 1)
-            per = 1;
-        blocks = std::min(per * g.num_sms, kMsMaxBlocks);
+        for (int k = 0; k < 2; k++) {
+            const void *f = k ? (const void *)k_msbfs<2> : (const void *)k_msbfs<1>;
+            int per = 0;
+            GB_CUDA_TRY(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kMsSmem));
+            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, f, kBlock, kMsSmem) != cudaSuccess || per < 1)
+                per = 1;
+            blocks[k] = std::min(per * g.num_sms, kMsMaxBlocks);
+        }
     }
     MsParams P;
     P.brow = g.brow; P.badj = g.badj; P.borig = g.borig; P.bord = g.bord; P.brank = g.brank;
@@ -927,15 +952,17 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
     P.tkey = o.tkey; P.qv = o.qv; P.parq = o.parq; P.pp = o.pp; P.rec = o.rec; P.crec = o.crec; P.irec = o.irec;
     P.lvl = o.lvl; P.vbase = o.vbase; P.depth = o.depth; P.maxd = o.maxd;
     P.prof = ws.msprof;
-    GB_CUDA_TRY(cudaMemsetAsync(ws.vis, 0, sizeof(unsigned long long) * 2 * (size_t)g.n, st));
-    GB_CUDA_TRY(cudaMemsetAsync(ws.fr, 0, sizeof(unsigned long long) * 2 * (size_t)g.n, st));
+    GB_CUDA_TRY(cudaMemsetAsync(ws.vis, 0, sizeof(unsigned long long) * S * (size_t)g.n, st));
+    GB_CUDA_TRY(cudaMemsetAsync(ws.fr, 0, sizeof(unsigned long long) * S * (size_t)g.n, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.fbm, 0, sizeof(uint32_t) * 6 * (size_t)P.nwords, st));
     GB_CUDA_TRY(cudaMemsetAsync(ws.msflag, 0, sizeof(int32_t) * 8, st));
     const int64_t work = std::max<int64_t>((int64_t)B * g.nbig, g.niso);
-    k_ms_roots<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, 8192)), 256, 0, st>>>(P);
+    const unsigned rgrid = (unsigned)std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, 8192));
+    if (S == 2) k_ms_roots<2><<<rgrid, 256, 0, st>>>(P);
+    else k_ms_roots<1><<<rgrid, 256, 0, st>>>(P);
     ++*launches;
     void *args[] = {&P};
-    cudaError_t e = cudaLaunchCooperativeKernel((const void *)k_msbfs, dim3(blocks), dim3(kBlock), args, kMsSmem, st);
+    cudaError_t e = cudaLaunchCooperativeKernel(kern, dim3(blocks[S - 1]), dim3(kBlock), args, kMsSmem, st);
     if (e != cudaSuccess) {
         set_error(std::string("cooperative launch (msbfs): ") + cudaGetErrorString(e));
         return GB_ECUDA;
