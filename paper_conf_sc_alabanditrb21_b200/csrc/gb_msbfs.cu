@@ -180,10 +180,13 @@ __device__ __forceinline__ W2 ms_chunk_or(const MsParams &P, const unsigned long
     return W2{warp_or64(acc.a), warp_or64(acc.b)};
 }
 
+// 64-bit warp minimum as two 32-bit redux.sync reductions (lexicographic:
+// the high words, then the low words of the lanes holding the high minimum)
 __device__ __forceinline__ unsigned long long warp_min64(unsigned long long v) {
-#pragma unroll
-    for (int d = 16; d; d >>= 1) v = min(v, __shfl_xor_sync(0xFFFFFFFFu, v, d));
-    return v;
+    const uint32_t hi = (uint32_t)(v >> 32);
+    const uint32_t mh = __reduce_min_sync(0xFFFFFFFFu, hi);
+    const uint32_t ml = __reduce_min_sync(0xFFFFFFFFu, hi == mh ? (uint32_t)v : 0xFFFFFFFFu);
+    return ((unsigned long long)mh << 32) | ml;
 }
 
 // best parent keys of vertex ow over the slots [s0, s1) for the trees in

@@ -85,9 +85,10 @@ __device__ __forceinline__ uint32_t tb_incl_scan32(uint32_t v) {
 }
 
 __device__ __forceinline__ unsigned long long tb_warp_min64(unsigned long long v) {
-#pragma unroll
-    for (int d = 16; d; d >>= 1) v = min(v, __shfl_xor_sync(0xFFFFFFFFu, v, d));
-    return v;
+    const uint32_t hi = (uint32_t)(v >> 32);
+    const uint32_t mh = __reduce_min_sync(0xFFFFFFFFu, hi);
+    const uint32_t ml = __reduce_min_sync(0xFFFFFFFFu, hi == mh ? (uint32_t)v : 0xFFFFFFFFu);
+    return ((unsigned long long)mh << 32) | ml;
 }
 
 // parent | neg << 31 as an internal id (keys carry the original id, R4)
