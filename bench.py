@@ -290,6 +290,7 @@ def main():
         # rank counts and the NCCL transport in the log (init lines only)
         os.environ.setdefault("NCCL_DEBUG", "INFO")
         os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+        os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")   # stdout carries the one JSON line
     import torch
     import torch.distributed as dist
     from paper_conf_sc_alabanditrb21_b200 import graphb
@@ -370,7 +371,7 @@ def main():
     dom_ms_per_launch = ph[dom] / dom_launches
     peak, peak_src = load_peaks()
     achieved = dom_bytes_per_launch / (dom_ms_per_launch / 1000.0) / 1e9
-    bfs_kernel = "k_tbfs" if any(kv.replace(" ", "") == "bfs=0" for kv in args.opt) else "k_msbfs"
+    bfs_kernel = "k_msbfs"
     opts = {kv.replace(" ", "").split("=")[0]: kv.replace(" ", "").split("=")[1] for kv in args.opt}
     walk_kernel = {0: "k_cycles_irec" if opts.get("jump", "1") == "1" else "k_cycles_jump",
                    1: "k_cycles_descent", 2: "k_cycles_paper"}[args.walk]

@@ -12,7 +12,7 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libgraphb.so")
 HEADER = os.path.join(os.path.dirname(HERE), "include", "graphb.h")
-SOURCES = ["gb_ingest.cu", "gb_msbfs.cu", "gb_tbfs.cu", "gb_tree.cu", "gb_cycle.cu", "gb_harary.cu", "gb_wilson.cu",
+SOURCES = ["gb_ingest.cu", "gb_msbfs.cu", "gb_tree.cu", "gb_cycle.cu", "gb_harary.cu", "gb_wilson.cu",
            "gb_api.cu"]
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
               "-Xcompiler", "-fPIC", "-shared"]

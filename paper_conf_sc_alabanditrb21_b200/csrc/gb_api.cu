@@ -60,9 +60,6 @@ struct Options {
     int64_t wilson = 0;      // sampler 1: 0 one thread per tree (W trees at once), 1 parallel cycle popping
     int64_t harary = 0;      // 1: Harary sides by the L224 procedure (gb_harary.cu)
     int64_t jump = 1;        // walk 0: levels per ancestor record of the cycle walk (1, 2, 4)
-    int64_t bfs = 1;         // 1 multi-source BFS (gb_msbfs.cu, default), 0 tree-parallel pull BFS (gb_tbfs.cu)
-    int64_t bfs_group = 4;   // bfs 0: trees per BFS launch (1..kTbMax)
-    int64_t push_k = 4;      // bfs 0: a level pushes while frontier slots * push_k < unvisited slots
 };
 
 struct Stats {
@@ -114,7 +111,7 @@ static void free_ws(Workspace &w) {
                     w.parq, w.offq, w.szq, w.pp, w.rec, w.irec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
                     w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof,
-                    w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey, w.tbm, w.tbhbest, w.tbhpos, w.tbhlev,
+                    w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey,
                     w.ptbase, w.ptnbr, w.ptrng};
     for (void *p : ptrs) if (p) cudaFree(p);
     w = Workspace();
@@ -122,14 +119,6 @@ static void free_ws(Workspace &w) {
 
 static void free_graph(Graph &g) {
     g = Graph();   // the arrays live in the persistent arena
-}
-
-static BfsOpts bfs_opts() {
-    BfsOpts b;
-    b.kind = (int)S.opt.bfs;
-    b.group = (int)S.opt.bfs_group;
-    b.push_k = (int)S.opt.push_k;
-    return b;
 }
 
 // record layout: 0 = records by internal id (walk 0, one level per record),
@@ -176,22 +165,7 @@ static int ensure_workspace(int B, bool descent) {
     ALLOC(w.msflag, 8);
     ALLOC(w.mscnt, (int64_t)kMsBatch * 2048);
     ALLOC(w.fbm, 6 * ((n + 31) / 32));
-    {   // tree-parallel BFS: bitmaps and hub tables of kTbMax trees
-        const int64_t G = kTbMax, nh = std::max<int64_t>(g.nmulti, 1);
-        ALLOC(w.tbm, (G * 6 + 1) * ((n + 31) / 32));
-        ALLOC(w.tbhbest, G * nh);
-        ALLOC(w.tbhpos, G * nh);
-        ALLOC(w.tbhlev, G * nh);
-        if (cudaMemset(w.tbhbest, 0xFF, sizeof(unsigned long long) * G * nh) != cudaSuccess ||
-            cudaMemset(w.tbhpos, 0xFF, sizeof(uint32_t) * G * nh) != cudaSuccess ||
-            cudaMemset(w.tbhlev, 0, sizeof(uint32_t) * G * nh) != cudaSuccess) {
-            set_error("memset (tbfs hub tables) failed");
-            free_ws(S.ws);
-            return GB_ECUDA;
-        }
-        w.tbg = kTbMax;
-    }
-    ALLOC(w.qv, Bn);
+        ALLOC(w.qv, Bn);
     ALLOC(w.lvl, (int64_t)B * (n + 2));
     ALLOC(w.vbase, (int64_t)B * (n + 2));
     ALLOC(w.parq, Bn);
@@ -397,7 +371,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     T.batch_used = B;
     T.group_used = G;
     T.sub_used = auto_sub(B);
-    T.bfs_group_used = S.opt.sampler != 0 ? 1 : S.opt.bfs == 1 ? B : std::min<int64_t>(B, S.opt.bfs_group);
+    T.bfs_group_used = S.opt.sampler != 0 ? 1 : B;
     std::vector<cudaEvent_t> &evs = T.evs;
     const bool timing = S.opt.timing != 0;
     int64_t done = 0;
@@ -448,8 +422,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
             given = reinterpret_cast<const int32_t *>(S.ws.wseq) + j * S.g.n;
         }
         rc = run_batch_tree(S.g, S.ws, nb, given, st, &T.launches, ev, descent, auto_sub(nb),
-                            (int)S.opt.recpass, (size_t)S.opt.persist, given ? 0 : (int)S.opt.sampler,
-                            bfs_opts());
+                            (int)S.opt.recpass, (size_t)S.opt.persist, given ? 0 : (int)S.opt.sampler);
         if (rc) return rc;
         if (ev) GB_CUDA_TRY(cudaEventRecord(ev[4], st));
         rc = run_batch_cycles(S.g, S.ws, nb, G, (int)S.opt.walk, st, &T.launches, jump, (int)S.opt.desc_linear,
@@ -506,7 +479,7 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
         d_given = reinterpret_cast<const int32_t *>(S.ws.wseq);
     }
     rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk >= 1, 1,
-                        0, 0, d_given ? 0 : (int)S.opt.sampler, bfs_opts());
+                        0, 0, d_given ? 0 : (int)S.opt.sampler);
     if (rc) return rc;
     if (user_tree) {
         unsigned long long vis = 0;
@@ -691,18 +664,7 @@ int gb_set_option(const char *key, int64_t value) {
         S.opt.sampler = value;
     }
     else if (!strcmp(key, "recpass")) S.opt.recpass = value != 0;
-    else if (!strcmp(key, "bfs")) {
-        if (value != 0 && value != 1) { set_error("bfs must be 0 (tree-parallel) or 1 (multi-source)"); return GB_EINVAL; }
-        S.opt.bfs = value;
-    }
-    else if (!strcmp(key, "bfs_group")) {
-        if (value < 1 || value > kTbMax) { set_error("bfs_group must be 1..16"); return GB_EINVAL; }
-        S.opt.bfs_group = value;
-    }
-    else if (!strcmp(key, "push_k")) {
-        if (value < 0 || value > 1024) { set_error("push_k must be 0..1024"); return GB_EINVAL; }
-        S.opt.push_k = value;
-    }
+
     else if (!strcmp(key, "jump")) {
         if (value != 1 && value != 2 && value != 4) { set_error("jump must be 1, 2 or 4"); return GB_EINVAL; }
         S.opt.jump = value;

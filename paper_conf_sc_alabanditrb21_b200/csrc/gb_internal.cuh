@@ -18,7 +18,6 @@ constexpr int kBlock = 256;                  // threads per CTA of the cooperati
 constexpr int kMsBatch = 128;                // trees per multi-source BFS (one bit each, two 64-bit halves)
 constexpr int kLight = 8;                    // BFS: degree <= kLight -> one lane per vertex
 constexpr int kChunk = 256;                  // BFS: slots per warp work item of a heavier vertex
-constexpr int kTbMax = 16;                   // tree-parallel BFS: trees per launch (per-tree bitmaps)
 
 // ---------------------------------------------------------------------------
 // Counter-based hash: SplitMix64 finaliser and its inverse (R4).
@@ -187,12 +186,6 @@ struct Workspace {
                                         // [4..6] frontier sizes (levels mod 3)
     uint32_t *mscnt = nullptr;          // [128][2048] per-block discovery counts
     unsigned long long *msprof = nullptr;  // [256][4] BFS phase timestamps (option "msprof")
-    // tree-parallel BFS state (gb_tbfs.cu), G <= kTbMax trees per launch
-    uint32_t *tbm = nullptr;            // [G][6][ceil(n/32)] per-tree bitmaps + [ceil(n/32)] "finished"
-    unsigned long long *tbhbest = nullptr; // [G][nmulti] hub parent keys
-    uint32_t *tbhpos = nullptr;         // [G][nmulti] hub list positions
-    uint32_t *tbhlev = nullptr;         // [G][nmulti] hub discovery level + 2
-    int tbg = 0;                        // G the buffers hold
     uint32_t *fbm = nullptr;            // [6][ceil(n/32)] frontier bitmaps (3), finished bitmap,
                                         // two push bitmaps (direction optimisation)
     uint32_t *s1 = nullptr;    // [B][ncomp] #vertices with pi = 1 per component
@@ -263,15 +256,9 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr,
            const int32_t *h_col, const int8_t *h_sign, cudaStream_t st,
            int64_t *launches);
 
-struct BfsOpts {
-    int kind = 1;     // 1 multi-source BFS (gb_msbfs.cu), 0 tree-parallel pull BFS (gb_tbfs.cu)
-    int group = 4;    // kind 0: trees per launch
-    int push_k = 4;   // kind 0: a level pushes while frontier slots * push_k < unvisited slots
-};
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
                    cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub,
-                   int recpass = 0, size_t persist = 0, int sampler = 0,
-                   const BfsOpts &bfs = BfsOpts());
+                   int recpass = 0, size_t persist = 0, int sampler = 0);
 
 // f.3: uniform random spanning forest of tree ws.tkey[0] (Wilson by parallel
 // cycle popping, gb_wilson.cu) -> parent (-1 at the roots)
@@ -296,9 +283,7 @@ struct MsBfsOut {
 };
 int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStream_t st,
               int64_t *launches);
-// tree-parallel pull BFS (gb_tbfs.cu): the same outputs, G trees per launch
-int run_tbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStream_t st,
-             int64_t *launches, int G, int push_k);
+
 
 int debug_tree_views(const Graph &g, Workspace &ws, bool descent, int32_t *d_parent,
                      int32_t *d_dist, int32_t *d_size, int32_t *d_pre, cudaStream_t st);

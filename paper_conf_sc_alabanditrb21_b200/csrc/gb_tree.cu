@@ -933,7 +933,7 @@ static int set_window(cudaStream_t st, void *base, size_t bytes, size_t persist)
 
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
                    cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub,
-                   int recpass, size_t persist, int sampler, const BfsOpts &bfs) {
+                   int recpass, size_t persist, int sampler) {
     if (descent || ws.irec_layout) recpass = 0;
     // co-resident grid sizes, recomputed when the device changes
     static int bfs_blocks = 0, up_blocks[2] = {0, 0}, down_blocks[2] = {0, 0}, blocks_dev = -1;
@@ -983,8 +983,7 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
         o.irec = (ws.irec_layout && !descent) ? ws.irec : nullptr;
         o.crec = descent ? ws.crec : nullptr;
         o.lvl = ws.lvl; o.vbase = ws.vbase; o.depth = ws.depth; o.maxd = ws.maxd; o.tkey = ws.tkey;
-        int rc = bfs.kind == 1 ? run_msbfs(g, ws, B, o, st, launches)
-                               : run_tbfs(g, ws, B, o, st, launches, bfs.group, bfs.push_k);
+        int rc = run_msbfs(g, ws, B, o, st, launches);
         if (rc) return rc;
     }
     GB_CUDA_TRY(cudaGetLastError());
