@@ -189,52 +189,6 @@ __device__ __forceinline__ unsigned long long warp_min64(unsigned long long v) {
     return ((unsigned long long)mh << 32) | ml;
 }
 
-// best parent keys of vertex ow over the slots [s0, s1) for the trees in
-// `want` (one warp, lane = slot): per window of 32 slots, for every tree
-// present, the lanes whose neighbour is a candidate hash it and the warp
-// takes the minimum; lane l keeps trees l (b0) and l + 32 (b1).  When the
-// chunk is the whole adjacency and fits one window, a tree with a single
-// candidate takes it without hashing (its key then has score 0, which only
-// matters for the decode).
-template <int S>
-__device__ __forceinline__ void ms_chunk_keys(const MsParams &P, const unsigned long long *F,
-                                              const uint32_t *bm, uint32_t s0, uint32_t s1,
-                                              unsigned long long want, uint32_t ow, const uint64_t *s_tk,
-                                              bool whole, unsigned long long &b0, unsigned long long &b1,
-                                              int h) {
-    const int lane = threadIdx.x & 31;
-    b0 = ~0ull;
-    b1 = ~0ull;
-    const bool one = whole && s1 - s0 <= 32;
-    for (uint32_t base = s0; base < s1; base += 32) {
-        const uint32_t j = base + lane;
-        uint32_t o = 0;
-        unsigned long long f = 0;
-        if (j < s1) {
-            const uint32_t a = __ldg(P.badj + j);
-            f = fr_word<S>(F, bm, a & kIdMask, h) & want;
-            if (f) o = __ldg(P.borig + j) | (a & kNegBit);
-        }
-        for (unsigned long long rem = warp_or64(f); rem; rem &= rem - 1) {
-            const int t = __ffsll((long long)rem) - 1;
-            const bool has = (f >> t) & 1ull;
-            const uint32_t bal = __ballot_sync(0xFFFFFFFFu, has);
-            unsigned long long key;
-            if (one && !(bal & (bal - 1))) {
-                const uint32_t par = __shfl_sync(0xFFFFFFFFu, o, __ffs(bal) - 1);
-                key = ((unsigned long long)(par & kIdMask) << 1) | (par >> 31);
-            } else {
-                key = has ? parent_key(s_tk[t], o & kIdMask, ow, o >> 31) : ~0ull;
-                key = warp_min64(key);
-            }
-            if (lane == (t & 31)) {
-                if (t < 32) b0 = min(b0, key);
-                else b1 = min(b1, key);
-            }
-        }
-    }
-}
-
 // per-warp scratch of the parent pass (dynamic shared memory)
 constexpr int kMultiCap = 512;           // multi-candidate pairs per round
 struct WarpScratch {
@@ -461,6 +415,79 @@ __device__ __forceinline__ void ms_item_parents(const MsParams &P, const unsigne
     }
     p0 = key_to_par(W.best[lane]);
     p1 = key_to_par(W.best[lane + 32]);
+    __syncwarp();
+}
+
+// Best parent keys of vertex ow over the slots [s0, s1) (a chunk of <= 256
+// slots of a heavy vertex or a hub) for the trees in `want` (half h); lane l
+// returns trees l (b0) and l + 32 (b1).  Per window of 32 slots (lane = slot)
+// the (slot, tree) candidate pairs are listed tree-major in shared memory,
+// hashed 32 at a time with every lane busy (the min-hash rule, reading R4),
+// and reduced by a segmented warp minimum over the runs of equal trees; the
+// run tails fold their minimum into the per-tree best of the chunk.
+template <int S>
+__device__ __forceinline__ void ms_chunk_keys(const MsParams &P, const unsigned long long *F,
+                                              const uint32_t *bm, uint32_t s0, uint32_t s1,
+                                              unsigned long long want, uint32_t ow, const uint64_t *s_tk,
+                                              WarpScratch &W, unsigned long long &b0, unsigned long long &b1,
+                                              int h) {
+    const int lane = threadIdx.x & 31;
+    const uint32_t lt = (1u << lane) - 1u;
+    uint16_t *pl = reinterpret_cast<uint16_t *>(W.ml);   // 2 * kMultiCap pairs: lane << 6 | tree
+    constexpr uint32_t kCap = 2 * kMultiCap;
+    W.best[lane] = ~0ull;
+    W.best[lane + 32] = ~0ull;
+    __syncwarp();
+    for (uint32_t base = s0; base < s1; base += 32) {
+        const uint32_t j = base + lane;
+        uint32_t o = 0;
+        unsigned long long f = 0;
+        if (j < s1) {
+            const uint32_t a = __ldg(P.badj + j);
+            f = fr_word<S>(F, bm, a & kIdMask, h) & want;
+            if (f) o = __ldg(P.borig + j) | (a & kNegBit);
+        }
+        W.lo[0][lane] = o;
+        unsigned long long rem = warp_or64(f);
+        while (rem) {
+            // list the pairs of as many trees as fit, tree-major
+            uint32_t np = 0;
+            for (; rem && np + 32 <= kCap; rem &= rem - 1) {
+                const int t = __ffsll((long long)rem) - 1;
+                const bool has = (f >> t) & 1ull;
+                const uint32_t bal = __ballot_sync(0xFFFFFFFFu, has);
+                if (has) pl[np + __popc(bal & lt)] = (uint16_t)((lane << 6) | t);
+                np += __popc(bal);
+            }
+            __syncwarp();
+            for (uint32_t r0 = 0; r0 < np; r0 += 32) {
+                const uint32_t p = r0 + lane;
+                const bool valid = p < np;
+                const uint32_t e = valid ? pl[p] : 0u;
+                const int t = valid ? (int)(e & 63) : 64 + lane;   // unique for idle lanes
+                unsigned long long key = ~0ull;
+                if (valid) {
+                    const uint32_t oo = W.lo[0][e >> 6];
+                    key = parent_key(s_tk[t], oo & kIdMask, ow, oo >> 31);
+                }
+                // segmented inclusive minimum over runs of equal t
+                const int tprev = __shfl_up_sync(0xFFFFFFFFu, t, 1);
+                const uint32_t starts = __ballot_sync(0xFFFFFFFFu, lane == 0 || tprev != t);
+                const int leader = 31 - __clz(starts & (lt | (1u << lane)));
+#pragma unroll
+                for (int d = 1; d < 32; d <<= 1) {
+                    const unsigned long long y = __shfl_up_sync(0xFFFFFFFFu, key, d);
+                    if (lane - d >= leader) key = min(key, y);
+                }
+                const bool tail = lane == 31 || ((starts >> (lane + 1)) & 1u);
+                if (valid && tail) W.best[t] = min(W.best[t], key);   // one tail per tree per round
+                __syncwarp();
+            }
+        }
+        __syncwarp();
+    }
+    b0 = W.best[lane];
+    b1 = W.best[lane + 32];
     __syncwarp();
 }
 
@@ -794,7 +821,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                             ms_item_parents<S>(P, F, bm, it.y, s1, nw, ow, s_tk + tb, W, p0, p1, h);
                         } else {
                             unsigned long long b0, b1;
-                            ms_chunk_keys<S>(P, F, bm, it.y, s1, nw, ow, s_tk + tb, true, b0, b1, h);
+                            ms_chunk_keys<S>(P, F, bm, it.y, s1, nw, ow, s_tk + tb, W, b0, b1, h);
                             p0 = key_to_par(b0);
                             p1 = key_to_par(b1);
                         }
@@ -849,7 +876,7 @@ __global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
                     const unsigned long long want = h ? want2.b : want2.a;
                     if (!want) continue;
                     unsigned long long b0, b1;
-                    ms_chunk_keys<S>(P, F, bm, it.y, e1, want, __ldg(P.bord + hi), s_tk + 64 * h, false, b0, b1, h);
+                    ms_chunk_keys<S>(P, F, bm, it.y, e1, want, __ldg(P.bord + hi), s_tk + 64 * h, W, b0, b1, h);
                     if (b0 != ~0ull) atomicMin(P.hbest + (size_t)hi * kMsBatch + 64 * h + lane, b0);
                     if (b1 != ~0ull) atomicMin(P.hbest + (size_t)hi * kMsBatch + 64 * h + lane + 32, b1);
                 }
