@@ -110,7 +110,7 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
                           uint64_t *sum_cycle_len, int64_t *num_cycles);
 
 /* Options (before gb_balance*): "batch" trees per batch (0 = auto; at most
- * 64, the multi-source BFS width -- larger values are clamped to 64),
+ * 128, the multi-source BFS width -- larger values are clamped to 128),
  * "cycle_group" trees per cycle-kernel pass (0 = auto), "walk"
  * (0 = two-ended interval walk, 1 = Alg. 3 descent with warp ballots),
  * "timing" (1 = record per-phase CUDA events), "sub" (trees per labelling launch, 0 = auto), "msprof" (see gb_msbfs_profile),

@@ -190,7 +190,13 @@ __device__ __forceinline__ unsigned long long warp_min64(unsigned long long v) {
 }
 
 // per-warp scratch of the parent pass (dynamic shared memory)
-constexpr int kMultiCap = 512;           // multi-candidate pairs per round
+#ifndef GB_MS_MULTICAP
+#define GB_MS_MULTICAP 512
+#endif
+#ifndef GB_MS_MINBLOCKS
+#define GB_MS_MINBLOCKS 4
+#endif
+constexpr int kMultiCap = GB_MS_MULTICAP;   // multi-candidate pairs per round
 struct WarpScratch {
     uint32_t ml[kMultiCap];              // multi-candidate pairs: src << 14 | tree << 8 | slot mask
     unsigned long long pk[3][32];        // parent slot index k of (vertex lane, tree), bit-planes
@@ -580,7 +586,7 @@ __global__ void k_ms_roots(MsParams P) {
 //            then one more barrier.
 // ---------------------------------------------------------------------------
 template <int S>
-__global__ void __launch_bounds__(kBlock, 4) k_msbfs(MsParams P) {
+__global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
     cg::grid_group grid = cg::this_grid();
     __shared__ uint64_t s_tk[kMsBatch];
     __shared__ uint32_t s_cnt[kMsBatch], s_pos[kMsBatch], s_base[kMsBatch];
