@@ -374,7 +374,7 @@ def main():
     bfs_kernel = "k_msbfs"
     opts = {kv.replace(" ", "").split("=")[0]: kv.replace(" ", "").split("=")[1] for kv in args.opt}
     walk_kernel = {0: "k_cycles_irec" if opts.get("jump", "1") == "1" else "k_cycles_jump",
-                   1: "k_cycles_descent", 2: "k_cycles_paper"}[args.walk]
+                   1: "k_cycles_descent", 2: "k_cycles_paper", 3: "k_cycles_pclimb"}[args.walk]
     kernel_of = {"bfs": bfs_kernel, "bottom_up": "k_bottom_up", "top_down": "k_top_down",
                  "cycles": walk_kernel, "accumulate": "k_accumulate_edges", "init": "k_ms_roots"}
     traffic = ncu_traffic(args.config, kernel_of[dom], trees_in_step / dom_launches)
@@ -456,7 +456,8 @@ def main():
                        "cycles_per_tree": c_nt, "trees_per_gpu": T, "trees_total": total_trees,
                        "batch": phase["batch"], "cycle_group": phase["cycle_group"],
                        "bfs_trees_per_launch": phase["bfs_group"],
-                       "walk": "two-ended" if args.walk == 0 else "alg3-descent",
+                       "walk": {0: "two-ended interval climb", 1: "alg3-descent", 2: "paper edge lists",
+                                3: "pre-order climb"}[args.walk],
                        "avg_cycle_len": per_tree_sumk / max(1, c_nt),
                        "max_depth": phase["max_depth"],
                        "l2": "inputs larger than L2 (graph arrays > 126 MB)" if 16 * m > 126e6

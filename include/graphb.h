@@ -112,7 +112,12 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
 /* Options (before gb_balance*): "batch" trees per batch (0 = auto; at most
  * 128, the multi-source BFS width -- larger values are clamped to 128),
  * "cycle_group" trees per cycle-kernel pass (0 = auto), "walk"
- * (0 = two-ended interval walk, 1 = Alg. 3 descent with warp ballots),
+ * (0 = two-ended interval walk, 1 = Alg. 3 descent with warp ballots,
+ * 2 = the paper's partitioned two-word tree-edge lists (L238-L244) with a
+ * linear scan, 3 = pre-order climb: of the two current vertices the one with
+ * the larger pre climbs, 4-byte parent words indexed by pre), "desc_linear"
+ * (walk 1: 1 = linear int4 ballot rounds over the child starts, 0 = 32-ary
+ * pivots), "walk_ept" (walk 0: 1, 2 or 4 edges per thread),
  * "timing" (1 = record per-phase CUDA events), "sub" (trees per labelling launch, 0 = auto), "msprof" (see gb_msbfs_profile),
  * "recpass" (walk 0: 1 = pre-indexed records scattered in a pass after the
  * top-down pass, 0 = inside it), "jump" (walk 0: 1, 2 or 4 tree levels per

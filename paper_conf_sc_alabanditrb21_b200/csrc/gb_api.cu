@@ -48,7 +48,8 @@ void arena_free_all() {
 struct Options {
     int64_t batch = 0;       // 0 = auto
     int64_t cycle_group = 0; // 0 = auto
-    int64_t walk = 0;        // 0 two-ended, 1 Alg. 3 descent (child lists), 2 the paper's edge lists (L238-L244)
+    int64_t walk = 0;        // 0 two-ended, 1 Alg. 3 descent (child lists), 2 the paper's edge lists (L238-L244),
+                             // 3 pre-order climb (layout 2)
     int64_t desc_linear = 0; // walk 1: 1 = linear int4 ballot rounds over the child starts, 0 = 32-ary pivots
     int64_t walk_ept = 1;    // walk 0 (layout 0): edges per thread, climbed interleaved (1, 2, 4)
     int64_t timing = 0;
@@ -86,7 +87,7 @@ struct State {
     Graph g;
     Workspace ws;
     bool ws_descent = false;
-    bool ws_irec = false;
+    int ws_layout = -1;
     cudaStream_t stream = nullptr;
     int32_t *d_cnt = nullptr, *d_agree = nullptr;  // gb_balance's device counters
     int64_t cnt_cap_m = 0, cnt_cap_n = 0;          // their capacities (edges, vertices)
@@ -108,7 +109,7 @@ constexpr int64_t kStateSlots = 2 * kRecCap;  // open-addressing table of gb_clo
 
 static void free_ws(Workspace &w) {
     void *ptrs[] = {w.vst, w.qv, w.qs, w.qr, w.pkeyq, w.lvl, w.vbase, w.size, w.sz64,
-                    w.parq, w.offq, w.szq, w.pp, w.rec, w.irec, w.fbits, w.s1, w.tkey, w.depth,
+                    w.parq, w.offq, w.szq, w.pp, w.rec, w.irec, w.prec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
                     w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof,
                     w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey,
@@ -122,13 +123,18 @@ static void free_graph(Graph &g) {
 }
 
 // record layout: 0 = records by internal id (walk 0, one level per record),
-// 1 = pp + pre-indexed records (walk 1, option jump)
-static bool irec_layout() { return S.opt.walk == 0 && S.opt.jump == 1; }
+// 1 = pp + pre-indexed records (walks 1, 2, option jump), 2 = pp + 4-byte
+// pre-indexed parent words (walk 3)
+static int rec_layout() {
+    if (S.opt.walk == 3) return 2;
+    return (S.opt.walk == 0 && S.opt.jump == 1) ? 0 : 1;
+}
+static bool walk_descent() { return S.opt.walk == 1 || S.opt.walk == 2; }   // need the child lists
 
 static size_t per_tree_bytes(const Graph &g, bool descent) {
     const size_t n = (size_t)g.n;
     size_t b = 36 * n + 32 + 4 * (size_t)((g.m + 31) / 32) + 4 * (size_t)g.ncomp;
-    b += irec_layout() ? 16 * n : 12 * n;
+    b += rec_layout() == 0 ? 16 * n : rec_layout() == 1 ? 12 * n : 8 * n;
     if (descent) b += 24 * n;
     return b;
 }
@@ -144,8 +150,9 @@ static size_t per_tree_bytes(const Graph &g, bool descent) {
     } while (0)
 
 static int ensure_workspace(int B, bool descent) {
-    const bool irec = irec_layout();
-    if (S.ws.B >= B && descent == S.ws_descent && irec == S.ws_irec) return GB_OK;
+    const int layout = rec_layout();
+    const bool irec = layout == 0;
+    if (S.ws.B >= B && descent == S.ws_descent && layout == S.ws_layout) return GB_OK;
     B = std::max(B, S.ws.B);
     free_ws(S.ws);
     Workspace &w = S.ws;
@@ -173,6 +180,9 @@ static int ensure_workspace(int B, bool descent) {
     ALLOC(w.szq, Bn);
     if (irec) {
         ALLOC(w.irec, Bn);
+    } else if (layout == 2) {
+        ALLOC(w.pp, Bn);
+        ALLOC(w.prec, Bn);
     } else {
         ALLOC(w.pp, Bn);
         ALLOC(w.rec, Bn);
@@ -199,7 +209,7 @@ static int ensure_workspace(int B, bool descent) {
     w.B = B;
     w.n = n;
     S.ws_descent = descent;
-    S.ws_irec = irec;
+    S.ws_layout = layout;
     return GB_OK;
 }
 
@@ -267,7 +277,7 @@ static int auto_batch(int64_t ntrees) {
     // the multi-source BFS holds one bit per tree in a 128-bit word
     if (S.opt.batch > 0) return (int)std::min<int64_t>(S.opt.batch, kMsBatch);
     const size_t have = S.free_at_load;
-    int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, S.opt.walk >= 1));
+    int64_t bm = (int64_t)(0.5 * (double)have / (double)per_tree_bytes(S.g, walk_descent()));
     int64_t b = std::min<int64_t>({ntrees, (int64_t)kMsBatch, std::max<int64_t>(bm, 1)});
     return (int)std::max<int64_t>(b, 1);
 }
@@ -287,7 +297,7 @@ static int auto_sub(int B) {
 static int auto_group(int B) {
     if (S.opt.cycle_group > 0) return (int)std::min<int64_t>(S.opt.cycle_group, B);
     // keep the labels of the trees walked together L2-resident (~48 MB)
-    double per = (4.0 + 8.0 * (S.opt.walk == 0 ? S.opt.jump : 1)) * (double)S.g.n;
+    double per = (S.opt.walk == 3 ? 8.0 : 4.0 + 8.0 * (S.opt.walk == 0 ? S.opt.jump : 1)) * (double)S.g.n;
     int g = (int)std::max(1.0, std::floor(48.0e6 / per));
     return std::max(1, std::min(g, B));
 }
@@ -345,14 +355,14 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     T.pending = true;
     const int64_t K = t_end > t_begin ? (t_end - t_begin + stride - 1) / stride : 0;
     if (K == 0) return GB_OK;
-    const bool descent = S.opt.walk >= 1;   // walks 1 and 2 need the child lists
+    const bool descent = walk_descent();   // walks 1 and 2 need the child lists
     int B = auto_batch(K);
     // walk 1 keeps child lists of a whole batch in one 32-bit index space
     if (descent) B = (int)std::min<int64_t>(B, std::max<int64_t>(1, ((1ll << 32) - 1) / S.g.n));
     int rc = ensure_workspace(B, descent);
     if (rc) return rc;
     const int G = auto_group(B);
-    const int jump = descent ? 1 : (int)S.opt.jump;
+    const int jump = S.opt.walk == 0 ? (int)S.opt.jump : 1;
     if (jump > 1 && S.ws.jrec_cap < G * jump) {
         if (S.ws.jrec) cudaFree(S.ws.jrec);
         S.ws.jrec = nullptr;
@@ -460,7 +470,7 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
     Stats &T = S.st;
     drop_events(T);
     T = Stats();
-    int rc = ensure_workspace(1, S.opt.walk >= 1);
+    int rc = ensure_workspace(1, walk_descent());
     if (rc) return rc;
     cudaStream_t st = S.stream;
     k_tree_keys<<<1, kMaxBatch, 0, st>>>(S.ws.tkey, 1, seed, t, 1);
@@ -478,7 +488,7 @@ static int run_single_tree(int64_t t, uint64_t seed, const int32_t *d_given) {
         if (rc) return rc;
         d_given = reinterpret_cast<const int32_t *>(S.ws.wseq);
     }
-    rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, S.opt.walk >= 1, 1,
+    rc = run_batch_tree(S.g, S.ws, 1, d_given, st, &T.launches, nullptr, walk_descent(), 1,
                         0, 0, d_given ? 0 : (int)S.opt.sampler);
     if (rc) return rc;
     if (user_tree) {
@@ -645,7 +655,7 @@ int gb_set_option(const char *key, int64_t value) {
     if (!strcmp(key, "batch")) { if (value < 0) return GB_EINVAL; S.opt.batch = value; }
     else if (!strcmp(key, "cycle_group")) { if (value < 0) return GB_EINVAL; S.opt.cycle_group = value; }
     else if (!strcmp(key, "walk")) {
-        if (value < 0 || value > 2) { set_error("walk must be 0 (two-ended), 1 (Alg. 3 descent) or 2 (paper edge lists)"); return GB_EINVAL; }
+        if (value < 0 || value > 3) { set_error("walk must be 0 (two-ended), 1 (Alg. 3 descent), 2 (paper edge lists) or 3 (pre-order climb)"); return GB_EINVAL; }
         S.opt.walk = value;
     }
     else if (!strcmp(key, "desc_linear")) S.opt.desc_linear = value != 0;
@@ -733,7 +743,7 @@ int gb_tree_debug(int64_t t, uint64_t seed, int32_t *parent, int32_t *dist, int3
     const int64_t n = S.g.n;
     int32_t *d_tmp = nullptr;
     GB_CUDA_TRY(cudaMalloc(&d_tmp, sizeof(int32_t) * 4 * n));
-    rc = debug_tree_views(S.g, S.ws, S.opt.walk >= 1, d_tmp, d_tmp + n, d_tmp + 2 * n, d_tmp + 3 * n, S.stream);
+    rc = debug_tree_views(S.g, S.ws, walk_descent(), d_tmp, d_tmp + n, d_tmp + 2 * n, d_tmp + 3 * n, S.stream);
     if (rc) { cudaFree(d_tmp); return rc; }
     std::vector<int32_t> h(4 * n);
     cudaError_t ce = cudaMemcpy(h.data(), d_tmp, sizeof(int32_t) * 4 * n, cudaMemcpyDeviceToHost);

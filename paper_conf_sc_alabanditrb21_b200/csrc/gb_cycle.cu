@@ -35,6 +35,7 @@ struct CycleParams {
     const uint32_t *pp;    // [B][n] pre | pi<<31
     const uint2 *rec;      // [B][n] pre-indexed {up | neg<<31, size}                (layout 1)
     const uint4 *irec;     // [B][n] by internal id {parent | neg, pre | pi, size, 0} (layout 0)
+    const uint32_t *prec;  // [B][n] pre-indexed parent word up | neg<<31       (layout 2)
     const uint2 *crec;     // [B][n] pre-indexed {child-list start, #children}
     const uint32_t *clist; // children pre IDs, per parent ascending
     uint32_t *fbits;       // [B][words]
@@ -142,6 +143,64 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_two_ended(CycleParams P)
             const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
             if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
             // per-tree cycle statistics and state signature
+            warp_stats(lane, g, k, cyc, flip != 0, e, s_k, s_c, s_sig);
+        }
+    }
+    __syncthreads();
+    flush_stats(P, s_k, s_c, s_sig);
+}
+
+// Walk 3 (layout 2): pre-order climb.  Ancestors precede their descendants
+// in pre order (pre c = pre p + offset, offset >= 1, Alg. 4), so of
+// two distinct vertices of one tree the one with the larger pre is not an
+// ancestor of the other: it lies strictly below their LCA, and climbing it is
+// always a step of the fundamental cycle; the two climbs meet exactly at the
+// LCA.  Only the pre labels steer the walk (the range ends are not read), and
+// a step is one 4-byte gather of prec[pre] = pre(parent) | neg<<31: the two
+// per-tree arrays (pp by internal id, prec by pre, 8 bytes per vertex) are
+// the walk's whole random-access working set.
+__global__ void __launch_bounds__(kCycleBlock) k_cycles_pclimb(CycleParams P) {
+    __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup], s_sig[kMaxGroup];
+    for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; s_sig[i] = 0; }
+    __syncthreads();
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t word = gw; word < P.words; word += nw) {
+        const int64_t e = word * 32 + lane;
+        const bool valid = e < P.m;
+        uint2 ed = valid ? __ldg(P.edges + e) : make_uint2(0, 0);
+        const uint32_t u = ed.x, v = ed.y & kIdMask, nege = ed.y >> 31;
+        for (int g = 0; g < P.G; g++) {
+            const size_t nb = (size_t)(P.b0 + g) * P.n;
+            const uint32_t *pp = P.pp + nb, *prec = P.prec + nb;
+            uint32_t flip = 0, k = 0;
+            bool cyc = false;
+            if (valid) {
+                uint32_t x = __ldg(pp + u) & kIdMask, y = __ldg(pp + v) & kIdMask;
+                uint32_t rx = __ldg(prec + x), ry = __ldg(prec + y);
+                // tree edge iff one endpoint is the other's parent (simple graph)
+                if ((rx & kIdMask) != y && (ry & kIdMask) != x) {
+                    cyc = true;
+                    uint32_t c = 0;
+                    k = 1;
+                    while (x != y) {
+                        if (x > y) {
+                            c ^= rx;
+                            x = rx & kIdMask;
+                            if (x != y) rx = __ldg(prec + x);
+                        } else {
+                            c ^= ry;
+                            y = ry & kIdMask;
+                            if (x != y) ry = __ldg(prec + y);
+                        }
+                        k++;
+                    }
+                    flip = (c >> 31) ^ nege;
+                }
+            }
+            const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
+            if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
             warp_stats(lane, g, k, cyc, flip != 0, e, s_k, s_c, s_sig);
         }
     }
@@ -664,11 +723,13 @@ int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, int walk,
                      cudaStream_t st, int64_t *launches, int jump, int linear, int ept) {
     CycleParams P;
     const bool descent = walk == 1, paper = walk == 2;
+    if (walk == 3 && !ws.prec) { set_error("walk 3 needs layout 2"); return GB_EINVAL; }
     if (walk != 0 || !ws.jrec) jump = 1;
     P.jrec = ws.jrec;
     P.edges = g.edges_i; P.n = g.n; P.m = g.m;
     P.pp = ws.pp; P.rec = ws.rec; P.crec = ws.crec; P.clist = ws.clist;
     P.irec = ws.irec;
+    P.prec = ws.prec;
     P.linear = linear;
     P.tbase = nullptr; P.tnbr = nullptr; P.trng = nullptr;
     const bool irec = ws.irec_layout && walk == 0;
@@ -709,6 +770,7 @@ int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, int walk,
         else if (irec && ept == 2) k_cycles_irec_m<2><<<grid_cap(P.words * 16, kCycleBlock, g.num_sms, 8), kCycleBlock, 0, st>>>(P);
         else if (irec && ept == 4) k_cycles_irec_m<4><<<grid_cap(P.words * 8, kCycleBlock, g.num_sms, 8), kCycleBlock, 0, st>>>(P);
         else if (irec) k_cycles_irec<<<grid, kCycleBlock, 0, st>>>(P);
+        else if (walk == 3) k_cycles_pclimb<<<grid, kCycleBlock, 0, st>>>(P);
         else if (descent) k_cycles_descent<<<grid, kCycleBlock, 0, st>>>(P);
         else if (jump == 2) k_cycles_jump<2><<<grid, kCycleBlock, 0, st>>>(P);
         else if (jump == 4) k_cycles_jump<4><<<grid, kCycleBlock, 0, st>>>(P);

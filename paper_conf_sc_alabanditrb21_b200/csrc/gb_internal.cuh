@@ -163,6 +163,7 @@ struct Workspace {
     uint32_t *pp = nullptr;    // v: pre | pi<<31  (pi = root-path parity)      [layout 1]
     uint2 *rec = nullptr;      // pre: {up pre | neg<<31, size}                  [layout 1]
     uint4 *irec = nullptr;     // v: {parent | neg<<31, pre | pi<<31, size, 0}   [layout 0]
+    uint32_t *prec = nullptr;  // pre: up pre | neg<<31 (4 bytes)                [layout 2, walk 3]
     bool irec_layout = false;  // layout 0 (walk 0 with one level per record, the default):
                                // records indexed by internal vertex id, written by the
                                // top-down pass itself; layout 1 (walk 1, option jump):
@@ -276,6 +277,7 @@ struct MsBfsOut {
     uint32_t *qv, *parq, *pp;
     uint2 *rec, *crec;
     uint4 *irec;
+    uint32_t *prec;
     uint64_t *lvl;
     uint32_t *vbase;
     int32_t *depth, *maxd;
@@ -289,7 +291,7 @@ int debug_tree_views(const Graph &g, Workspace &ws, bool descent, int32_t *d_par
                      int32_t *d_dist, int32_t *d_size, int32_t *d_pre, cudaStream_t st);
 
 // walk: 0 two-ended, 1 Alg. 3 descent over child lists, 2 the paper's
-// partitioned two-word edge lists (linear scan)
+// partitioned two-word edge lists (linear scan), 3 pre-order climb (layout 2)
 int run_batch_cycles(const Graph &g, Workspace &ws, int B, int group, int walk,
                      cudaStream_t st, int64_t *launches, int jump = 1, int linear = 0, int ept = 1);
 

@@ -61,6 +61,7 @@ struct MsParams {
     uint32_t *qv, *parq, *pp;
     uint2 *rec, *crec;
     uint4 *irec;
+    uint32_t *prec;
     uint64_t *lvl;
     uint32_t *vbase;
     int32_t *depth, *maxd;
@@ -531,7 +532,8 @@ __global__ void k_ms_roots(MsParams P) {
             for (int b = 0; b < P.B; b++) {
                 const size_t nb = (size_t)b * P.n;
                 P.pp[nb + i] = pre;
-                P.rec[nb + pre] = make_uint2(pre, 1u);
+                if (P.prec) P.prec[nb + pre] = pre;
+                else P.rec[nb + pre] = make_uint2(pre, 1u);
                 if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
             }
         }
@@ -985,7 +987,7 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
     P.fcnt = reinterpret_cast<uint32_t *>(ws.msflag + 4);
     P.push_div = 32;   // measured on C3: 32 and 128 equal (bfs 59.0 ms / 100 trees), 8 worse (61.3)
     P.flag = ws.msflag; P.mscnt = ws.mscnt;
-    P.tkey = o.tkey; P.qv = o.qv; P.parq = o.parq; P.pp = o.pp; P.rec = o.rec; P.crec = o.crec; P.irec = o.irec;
+    P.tkey = o.tkey; P.qv = o.qv; P.parq = o.parq; P.pp = o.pp; P.rec = o.rec; P.crec = o.crec; P.irec = o.irec; P.prec = o.prec;
     P.lvl = o.lvl; P.vbase = o.vbase; P.depth = o.depth; P.maxd = o.maxd;
     P.prof = ws.msprof;
     GB_CUDA_TRY(cudaMemsetAsync(ws.vis, 0, sizeof(unsigned long long) * S * (size_t)g.n, st));

@@ -54,6 +54,7 @@ struct TreeParams {
     uint32_t *pp;
     uint2 *rec;
     uint4 *irec;                 // layout 0: {parent | neg, pre | pi, size, 0} by internal id
+    uint32_t *prec;              // layout 2: up pre | neg by pre (pp holds pre | pi by internal id)
     uint32_t *s1;
     const uint64_t *tkey;
     int32_t *depth, *maxd;
@@ -131,7 +132,8 @@ __device__ __forceinline__ void place_root(const TreeParams &P, int b, int64_t C
             P.irec[nb + ri] = make_uint4(ri, pre, 1u, 0u);
         } else {
             P.pp[nb + ri] = pre;
-            P.rec[nb + pre] = make_uint2(pre, 1u);
+            if (P.prec) P.prec[nb + pre] = pre;
+            else P.rec[nb + pre] = make_uint2(pre, 1u);
             if (P.crec) P.crec[nb + pre] = make_uint2(0u, 0u);
         }
         if (P.visited) atomicAdd(P.visited + b, 1ull);
@@ -690,6 +692,10 @@ __global__ void __launch_bounds__(kBlock, 4) k_top_down(TreeParams P) {
                     if (P.irec) {
                         // layout 0: the record by internal id, complete here
                         P.irec[nbk[k] + x[k]] = make_uint4(pq[k], pre | pi, szx[k], 0u);
+                    } else if (P.prec) {
+                        // layout 2: pre | pi by internal id, the parent word by pre
+                        P.pp[nbk[k] + x[k]] = pre | pi;
+                        P.prec[nbk[k] + pre] = up | neg;
                     } else if (P.recpass) {
                         P.pp[nbk[k] + x[k]] = pre | pi;
                         GB_QST(P.parq + qi[k], up | neg);
@@ -738,6 +744,9 @@ __global__ void __launch_bounds__(kBlock, 4) k_top_down(TreeParams P) {
             }
             if (!kDescent && P.irec) {
                 P.irec[nb + x] = make_uint4(L == 0 ? x : (p | neg), pre | pi, szx, 0u);
+            } else if (!kDescent && P.prec) {
+                P.pp[nb + x] = pre | pi;
+                P.prec[nb + pre] = up | neg;
             } else if (!kDescent && P.recpass) {
                 P.pp[nb + x] = pre | pi;
                 P.parq[qi] = up | neg;
@@ -891,6 +900,7 @@ static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_
     P.cidxq = descent ? ws.cidxq : nullptr;
     P.pp = ws.pp; P.rec = ws.rec; P.s1 = ws.s1; P.tkey = ws.tkey; P.depth = ws.depth;
     P.irec = (ws.irec_layout && !descent) ? ws.irec : nullptr;
+    P.prec = descent ? nullptr : ws.prec;
     P.maxd = ws.maxd; P.given = given;
     P.cstart = descent ? ws.cstart : nullptr;
     P.clist = descent ? ws.clist : nullptr;
@@ -904,6 +914,7 @@ static TreeParams make_params(const Graph &g, Workspace &ws, int B, const int32_
         if (P.pp) P.pp += nb;
         if (P.rec) P.rec += nb;
         if (P.irec) P.irec += nb;
+        if (P.prec) P.prec += nb;
         if (P.size) P.size += (size_t)b0 * P.szn;
         if (P.sz64) P.sz64 += nb;
         if (P.cidxq) P.cidxq += nb;
@@ -934,7 +945,7 @@ static int set_window(cudaStream_t st, void *base, size_t bytes, size_t persist)
 int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_parent,
                    cudaStream_t st, int64_t *launches, cudaEvent_t *ev, bool descent, int sub,
                    int recpass, size_t persist, int sampler) {
-    if (descent || ws.irec_layout) recpass = 0;
+    if (descent || ws.irec_layout || ws.prec) recpass = 0;
     // co-resident grid sizes, recomputed when the device changes
     static int bfs_blocks = 0, up_blocks[2] = {0, 0}, down_blocks[2] = {0, 0}, blocks_dev = -1;
     if (blocks_dev != g.dev) {
@@ -981,6 +992,7 @@ int run_batch_tree(const Graph &g, Workspace &ws, int B, const int32_t *given_pa
         MsBfsOut o;
         o.qv = ws.qv; o.parq = ws.parq; o.pp = ws.pp; o.rec = ws.rec;
         o.irec = (ws.irec_layout && !descent) ? ws.irec : nullptr;
+        o.prec = descent ? nullptr : ws.prec;
         o.crec = descent ? ws.crec : nullptr;
         o.lvl = ws.lvl; o.vbase = ws.vbase; o.depth = ws.depth; o.maxd = ws.maxd; o.tkey = ws.tkey;
         int rc = run_msbfs(g, ws, B, o, st, launches);

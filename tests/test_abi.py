@@ -58,13 +58,13 @@ def test_state_and_argument_errors_without_gpu():
     assert L.gb_load_csr(2, 2, rp.ctypes.data, col.ctypes.data, sg.ctypes.data) == graphb.GB_EINVAL
     assert L.gb_load_csr(2, 1, rp.ctypes.data, None, None) == graphb.GB_EINVAL
     assert L.gb_set_option(b"nope", 1) == graphb.GB_EINVAL
-    assert L.gb_set_option(b"walk", 3) == graphb.GB_EINVAL          # two-ended, Alg. 3, paper lists
+    assert L.gb_set_option(b"walk", 4) == graphb.GB_EINVAL          # two-ended, Alg. 3, paper lists, pre climb
     assert L.gb_set_option(b"graphs", 1) == graphb.GB_EINVAL        # not an option (never implemented)
     assert L.gb_set_option(b"sampler", 3) == graphb.GB_EINVAL      # BFS, uniform, DFS only
     assert L.gb_set_option(b"sampler", -1) == graphb.GB_EINVAL
     assert L.gb_set_option(b"jump", 3) == graphb.GB_EINVAL         # 1, 2 or 4 levels
     for k, v in [(b"sampler", 2), (b"wilson", 1), (b"harary", 1), (b"jump", 4), (b"recpass", 0),
-                 (b"walk", 2), (b"desc_linear", 1), (b"walk_ept", 4),
+                 (b"walk", 2), (b"walk", 3), (b"desc_linear", 1), (b"walk_ept", 4),
                  (b"batch", 128)]:
         assert L.gb_set_option(k, v) == 0
     assert L.gb_set_option(b"reset", 0) == 0

@@ -93,13 +93,13 @@ def test_c1_config_exact():
     assert st["trees"] == 1
 
 
-@pytest.mark.parametrize("walk", [0, 1, 2])
+@pytest.mark.parametrize("walk", [0, 1, 2, 3])
 def test_tree_stages_match_oracle(walk):
     g = graphgen.er(3000, 12000, 0.3, 4)
     check_tree_debug(g, 5, range(6), walk=walk)
 
 
-@pytest.mark.parametrize("walk,linear", [(0, 0), (1, 0), (1, 1), (2, 0)])
+@pytest.mark.parametrize("walk,linear", [(0, 0), (1, 0), (1, 1), (2, 0), (3, 0)])
 def test_power_law_hubs_multi_batch(walk, linear):
     """Hubs (Chung-Lu, children lists of thousands) + several batches + cycle
     groups smaller than a batch; walk 1 with 32-ary pivots and with linear
@@ -128,7 +128,7 @@ def test_msbfs_128_tree_pass():
     assert st["batch"] == 128 and st["batches"] == 2
 
 
-@pytest.mark.parametrize("walk", [1, 2])
+@pytest.mark.parametrize("walk", [0, 1, 2, 3])
 def test_paper_walks_on_forests_and_degenerate_trees(walk):
     """Walks 1 and 2 on a forest with isolated vertices (roots without a
     parent edge) and on a star (one hub with every vertex as a child)."""
@@ -229,7 +229,7 @@ def test_dfs_sampler_cloud(which):
     check_cloud(_uniform_graphs()[which], 5, 6, sampler=2)
 
 
-@pytest.mark.parametrize("sampler,walk,harary", [(1, 1, 0), (2, 1, 0), (1, 0, 1), (2, 0, 1)])
+@pytest.mark.parametrize("sampler,walk,harary", [(1, 1, 0), (2, 1, 0), (1, 0, 1), (2, 0, 1), (1, 3, 0), (2, 3, 1)])
 def test_samplers_with_descent_walk_and_l224_sides(sampler, walk, harary):
     """f.3 samplers combined with Alg. 3's descent walk (walk 1) and with the
     paper's L224 Harary procedure (f.2): still the oracle's cloud."""
