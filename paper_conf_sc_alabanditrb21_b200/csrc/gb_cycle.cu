@@ -89,6 +89,14 @@ __device__ __forceinline__ void flush_stats(const CycleParams &P, const unsigned
     }
 }
 
+// &base[i] as one mad.wide.u32 (i * 16 + base): the compiler otherwise widens
+// and masks the 31-bit id in 64-bit arithmetic (six instructions per step)
+__device__ __forceinline__ const uint4 *rec_at(const uint4 *base, uint32_t i) {
+    const uint4 *p;
+    asm("mad.wide.u32 %0, %1, 16, %2;" : "=l"(p) : "r"(i), "l"(base));
+    return p;
+}
+
 __device__ __forceinline__ bool is_anc(uint32_t a, uint32_t size_a, uint32_t t) {
     return (t - a) < size_a;  // a <= t <= a + size_a - 1 (unsigned wrap for t < a)
 }
@@ -231,7 +239,7 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_irec(CycleParams P) {
             uint32_t flip = 0, k = 0;
             bool cyc = false;
             if (valid) {
-                uint4 rx = __ldg(rec + u), ry = __ldg(rec + v);
+                uint4 rx = __ldg(rec_at(rec, u)), ry = __ldg(rec_at(rec, v));
                 // tree edge iff one endpoint is the other's parent (simple graph)
                 if ((rx.x & kIdMask) != v && (ry.x & kIdMask) != u) {
                     cyc = true;
@@ -242,13 +250,13 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_irec(CycleParams P) {
                     while (!(ax && ay)) {
                         if (!ax) {
                             c ^= rx.x;
-                            rx = __ldg(rec + (rx.x & kIdMask));
+                            rx = __ldg(rec_at(rec, rx.x & kIdMask));
                             k++;
                             ax = is_anc(rx.y & kIdMask, rx.z, py);
                         }
                         if (!ay) {
                             c ^= ry.x;
-                            ry = __ldg(rec + (ry.x & kIdMask));
+                            ry = __ldg(rec_at(rec, ry.x & kIdMask));
                             k++;
                             ay = is_anc(ry.y & kIdMask, ry.z, px);
                         }
