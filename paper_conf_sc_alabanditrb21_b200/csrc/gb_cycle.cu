@@ -304,8 +304,8 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_irec_m(CycleParams P) {
             bool ax[EPT], ay[EPT], cyc[EPT];
 #pragma unroll
             for (int j = 0; j < EPT; j++) {
-                rx[j] = valid[j] ? __ldg(rec + u[j]) : make_uint4(0, 0, 1, 0);
-                ry[j] = valid[j] ? __ldg(rec + v[j]) : make_uint4(0, 0, 1, 0);
+                rx[j] = valid[j] ? __ldg(rec_at(rec, u[j])) : make_uint4(0, 0, 1, 0);
+                ry[j] = valid[j] ? __ldg(rec_at(rec, v[j])) : make_uint4(0, 0, 1, 0);
             }
 #pragma unroll
             for (int j = 0; j < EPT; j++) {
@@ -324,12 +324,12 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_irec_m(CycleParams P) {
                 for (int j = 0; j < EPT; j++) {
                     if (!ax[j]) {
                         c[j] ^= rx[j].x;
-                        rx[j] = __ldg(rec + (rx[j].x & kIdMask));
+                        rx[j] = __ldg(rec_at(rec, rx[j].x & kIdMask));
                         k[j]++;
                     }
                     if (!ay[j]) {
                         c[j] ^= ry[j].x;
-                        ry[j] = __ldg(rec + (ry[j].x & kIdMask));
+                        ry[j] = __ldg(rec_at(rec, ry[j].x & kIdMask));
                         k[j]++;
                     }
                 }
