@@ -280,9 +280,23 @@ __global__ void k_slots(const uint32_t *__restrict__ rp, const int32_t *__restri
                         const uint32_t *__restrict__ uptr, const uint32_t *__restrict__ ebase,
                         uint32_t *__restrict__ adj, uint32_t *__restrict__ adj_eid,
                         uint2 *__restrict__ edges, uint32_t *err) {
-    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < slots;
-         j += (uint64_t)gridDim.x * blockDim.x) {
-        uint32_t u = row_of_slot(rp, n, (uint32_t)j);
+    // a warp takes 32 consecutive slots: the rows of its first and last slot
+    // by binary search over all rows, every lane's row by a search between them
+    const int lane = threadIdx.x & 31;
+    const uint64_t nwarp = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t base = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5 << 5; base < slots;
+         base += nwarp * 32) {
+        const uint64_t j = base + lane;
+        uint32_t r = 0;
+        if (lane == 0) r = row_of_slot(rp, n, (uint32_t)base);
+        if (lane == 31) r = row_of_slot(rp, n, (uint32_t)min(base + 31, slots - 1));
+        const uint32_t r0 = __shfl_sync(0xFFFFFFFFu, r, 0), r1 = __shfl_sync(0xFFFFFFFFu, r, 31);
+        if (j >= slots) continue;
+        uint32_t u = r0, hi = r1 + 1;  // rp[u] <= j < rp[hi]
+        while (hi - u > 1) {
+            const uint32_t mid = u + ((hi - u) >> 1);
+            if (__ldg(rp + mid) <= (uint32_t)j) u = mid; else hi = mid;
+        }
         int32_t v = col[j];
         int8_t s = sign[j];
         uint32_t e = 0;
@@ -328,18 +342,52 @@ __global__ void k_cc_init(int32_t *lab, int64_t n) {
         lab[v] = (int32_t)v;
 }
 
-__global__ void k_cc_hook(const uint2 *__restrict__ edges, int64_t m, int32_t *lab) {
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m;
-         e += (int64_t)gridDim.x * blockDim.x) {
-        uint2 ed = edges[e];
-        int32_t a = cc_find(lab, (int32_t)ed.x), b = cc_find(lab, (int32_t)(ed.y & kIdMask));
-        while (a != b) {
-            if (a < b) { int32_t t = a; a = b; b = t; }
-            int32_t old = atomicCAS(lab + a, a, b);
-            if (old == a) break;
-            a = cc_find(lab, old);
-            b = cc_find(lab, b);
-        }
+__device__ __forceinline__ void cc_hook(int32_t *lab, int32_t x, int32_t y) {
+    int32_t a = cc_find(lab, x), b = cc_find(lab, y);
+    while (a != b) {
+        if (a < b) { int32_t t = a; a = b; b = t; }
+        int32_t old = atomicCAS(lab + a, a, b);
+        if (old == a) break;
+        a = cc_find(lab, old);
+        b = cc_find(lab, b);
+    }
+}
+
+// Components in the manner of Afforest: every vertex is first hooked to its
+// first two neighbours (two cheap rounds that join almost all of a large
+// component), the largest component is identified from a sample, and only
+// the vertices outside it hook their remaining edges.  Hooking is still
+// "larger root under smaller", so every root is its component's minimum
+// vertex, as with the full edge pass.
+__global__ void k_cc_link(const uint32_t *__restrict__ rp, const uint32_t *__restrict__ adj, int64_t n,
+                          uint32_t k, int32_t *lab) {
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n;
+         u += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t j = __ldg(rp + u) + k;
+        if (j < __ldg(rp + u + 1)) cc_hook(lab, (int32_t)u, (int32_t)(__ldg(adj + j) & kIdMask));
+    }
+}
+
+__global__ void k_cc_compress(int32_t *lab, int64_t n) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+         v += (int64_t)gridDim.x * blockDim.x)
+        lab[v] = cc_find(lab, (int32_t)v);
+}
+
+__global__ void k_cc_sample(int32_t *lab, int64_t n, int32_t *out, int count) {
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < count) out[i] = cc_find(lab, (int32_t)(((uint64_t)i * 2654435761ull) % (uint64_t)n));
+}
+
+// the remaining edges (from neighbour k on) of every vertex outside component big
+__global__ void k_cc_rest(const uint32_t *__restrict__ rp, const uint32_t *__restrict__ adj, int64_t n,
+                          uint32_t k, int32_t big, int32_t *lab) {
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < n;
+         u += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t e = __ldg(rp + u + 1);
+        uint32_t j = __ldg(rp + u) + k;
+        if (j >= e || cc_find(lab, (int32_t)u) == big) continue;
+        for (; j < e; j++) cc_hook(lab, (int32_t)u, (int32_t)(__ldg(adj + j) & kIdMask));
     }
 }
 
@@ -510,6 +558,7 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
     int8_t *d_sign = nullptr;
     uint32_t *d_err = nullptr, *uptr = nullptr, *upc = nullptr, *ebase = nullptr,
              *tmp = nullptr, *flag = nullptr, *rank = nullptr;
+    std::vector<int32_t> smp;   // component sample (Afforest-style CC)
     int rc = GB_OK;
     uint32_t h_err = 0;
     size_t ntmp = scan_tmp_elems(std::max<int64_t>(n, 1));
@@ -572,7 +621,27 @@ int ingest(Graph &g, int64_t n, int64_t m, const int64_t *h_row_ptr, const int32
     k_cc_init<<<grid_for(n, 256, sms), 256, 0, st>>>(lab, n);
     ++*launches;
     if (m) {
-        k_cc_hook<<<grid_for(m, 256, sms), 256, 0, st>>>(g.edges, m, lab);
+        const int kSample = (int)std::min<int64_t>(1024, n);
+        for (uint32_t k = 0; k < 2; k++) {
+            k_cc_link<<<grid_for(n, 256, sms), 256, 0, st>>>(g.row_ptr, g.adj, n, k, lab);
+            k_cc_compress<<<grid_for(n, 256, sms), 256, 0, st>>>(lab, n);
+            *launches += 2;
+        }
+        int32_t *d_smp = reinterpret_cast<int32_t *>(flag);   // scratch until k_cc_finish
+        k_cc_sample<<<(kSample + 255) / 256, 256, 0, st>>>(lab, n, d_smp, kSample);
+        ++*launches;
+        smp.resize(kSample);
+        ING_TRY(cudaMemcpyAsync(smp.data(), d_smp, sizeof(int32_t) * kSample, cudaMemcpyDeviceToHost, st));
+        ING_TRY(cudaStreamSynchronize(st));
+        std::sort(smp.begin(), smp.end());
+        int32_t big = smp[0];
+        for (int i = 0, best = 0; i < kSample;) {
+            int k = i;
+            while (k < kSample && smp[k] == smp[i]) k++;
+            if (k - i > best) { best = k - i; big = smp[i]; }
+            i = k;
+        }
+        k_cc_rest<<<grid_for(n, 256, sms), 256, 0, st>>>(g.row_ptr, g.adj, n, 2, big, lab);
         ++*launches;
     }
     k_cc_finish<<<grid_for(n, 256, sms), 256, 0, st>>>(lab, n, flag, ebase);
