@@ -599,3 +599,40 @@ def test_c5_rmat26_capacity_and_sampled_cycles():
         assert tuple(int(x) for x in per1[0]) == (sk, nc, dep, sig)
         assert sha(cnt_d.cpu().numpy().astype("<u4")) == hc
         assert sha(agr_d.cpu().numpy().astype("<u4")) == ha
+
+
+def _sweep_case(i):
+    """Case i of the randomized sweep: a seeded graph family and size, a tree
+    count that straddles the 64- and 128-tree MS-BFS widths, and random
+    batching / walk options (none of them may change a result)."""
+    rng = np.random.default_rng(1000 + i)
+    kind = ["er", "chung_lu", "bipartite", "forest", "grid", "rmat"][i % 6]
+    n = int(rng.integers(40, 2500))
+    if kind == "er":
+        g = graphgen.er(n, int(n * rng.uniform(1.2, 4.0)), float(rng.uniform(0.0, 0.6)), 50 + i)
+    elif kind == "chung_lu":
+        g = graphgen.chung_lu(n, int(n * rng.uniform(2.0, 6.0)), max(8, n // 5), 2.2, float(rng.uniform(0.1, 0.5)),
+                              50 + i, lcc=bool(i % 2))
+    elif kind == "bipartite":
+        nu = n // 2
+        g = graphgen.bipartite_chung_lu(nu, n - nu, int(n * 2.2), 16, max(8, n // 6), 2.5, 2.1, 0.5, 50 + i)
+    elif kind == "forest":
+        g = graphgen.er(n, int(n * rng.uniform(0.3, 0.9)), 0.4, 50 + i)
+    elif kind == "grid":
+        g = graphgen.grid2d(int(rng.integers(3, 30)), int(rng.integers(3, 30)), float(rng.uniform(0, 0.5)), 50 + i)
+    else:
+        g = graphgen.rmat(int(rng.integers(7, 11)), 8, 0.3, 50 + i)
+    T = int(rng.choice([1, 2, 31, 63, 64, 65, 100, 127, 128, 129, 140]))
+    opts = {"walk": int(rng.choice([0, 0, 3, 1, 2])),
+            "batch": int(rng.choice([0, 0, 1, 7, 64, 65, 128])),
+            "cycle_group": int(rng.choice([0, 1, 3])),
+            "sub": int(rng.choice([0, 1, 3]))}
+    return g, T, int(rng.integers(1, 1 << 30)), opts
+
+
+@pytest.mark.parametrize("i", range(48))
+def test_randomized_sweep_bit_exact(i):
+    """48 seeded (graph, trees, seed, options) cases against the oracle: flip
+    counts, agree counts and every per-tree statistic bit for bit."""
+    g, T, seed, opts = _sweep_case(i)
+    check_cloud(g, T, seed, **opts)
