@@ -204,6 +204,7 @@ struct WarpScratch {
     uint32_t lo[kLight][32];             // candidate neighbour (original id) | neg << 31 (hashing)
     uint32_t li[kLight][32];             // the same neighbour as an internal id | neg << 31 (output)
     uint32_t ow[32];                     // original id of each lane's vertex
+    uint32_t iv[32];                     // internal id of each lane's vertex (emission)
     unsigned long long best[64];         // item parents: best key per tree (of the half)
 };
 constexpr size_t kMsSmem = sizeof(WarpScratch) * kMsWarps;
@@ -276,6 +277,7 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
         for (int k = 0; k < kLight; k++) c[k] = 0;
     }
     W.ow[lane] = ow;
+    W.iv[lane] = i;
     {   // slot-index planes of the single-candidate trees
         const unsigned long long sm = ~s2m;
         unsigned long long p0 = 0, p1 = 0, p2 = 0;
@@ -335,33 +337,45 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
     }
     __syncwarp();   // planes of every lane complete
     // emission: one shared-memory reservation per tree (lane t reserves the
-    // runs of trees t and t + 32, sized by the transposed discovery words),
-    // then tree by tree the discovering lanes write consecutive entries of the
-    // tree's level list (coalesced); the parent slot k comes from the planes
-    const unsigned long long mine_pk0 = W.pk[0][lane], mine_pk1 = W.pk[1][lane], mine_pk2 = W.pk[2][lane];
+    // runs of trees t and t + 32, sized by the transposed discovery words);
+    // lane t then lists its trees' (vertex lane, rank) pairs tree-major in
+    // shared memory, and the warp writes 32 listed entries per round, one per
+    // lane: consecutive lanes fill consecutive positions of a tree's level
+    // list, and the rounds number the pairs, not the trees
     const uint32_t nlo = transpose32((uint32_t)nw);
     const uint32_t nhi = transpose32((uint32_t)(nw >> 32));
     uint32_t blo = 0, bhi = 0;
     if (nlo) blo = s_base[lane] + atomicAdd(&s_pos[lane], (uint32_t)__popc(nlo));
     if (nhi) bhi = s_base[lane + 32] + atomicAdd(&s_pos[lane + 32], (uint32_t)__popc(nhi));
-    const uint32_t lt = (1u << lane) - 1u;
-#pragma unroll
-    for (int h = 0; h < 2; h++) {
-        for (uint32_t trees = __ballot_sync(0xFFFFFFFFu, (h ? nhi : nlo) != 0); trees; trees &= trees - 1) {
-            const int tl = __ffs(trees) - 1;
-            const int t = tl + 32 * h;
-            const uint32_t mask = __shfl_sync(0xFFFFFFFFu, h ? nhi : nlo, tl);
-            const uint32_t base = __shfl_sync(0xFFFFFFFFu, h ? bhi : blo, tl);
-            if ((mask >> lane) & 1u) {
-                const uint32_t k = (uint32_t)((mine_pk0 >> t) & 1ull) | ((uint32_t)((mine_pk1 >> t) & 1ull) << 1) |
-                                   ((uint32_t)((mine_pk2 >> t) & 1ull) << 2);
-                const size_t o = (size_t)(t + 64 * half) * P.n + base + __popc(mask & lt);
-                P.qv[o] = i;
-                P.parq[o] = W.li[k][lane];
-            }
+    uint32_t *sb = reinterpret_cast<uint32_t *>(W.best);   // list start per tree of the half
+    sb[lane] = blo;
+    sb[lane + 32] = bhi;
+    uint16_t *el = reinterpret_cast<uint16_t *>(W.ml);     // vertex lane | tree << 5 | rank << 11
+    constexpr uint32_t kCap = 2 * kMultiCap;
+    const uint32_t ne = (uint32_t)(__popc(nlo) + __popc(nhi));
+    const uint32_t eincl = warp_incl_scan32(ne);
+    const uint32_t etot = __shfl_sync(0xFFFFFFFFu, eincl, 31);
+    for (uint32_t r0 = 0; r0 < etot; r0 += kCap) {
+        uint32_t off = eincl - ne;
+        uint32_t r = 0;
+        for (uint32_t m = nlo; m && off < r0 + kCap; m &= m - 1, r++, off++)
+            if (off >= r0) el[off - r0] = (uint16_t)((__ffs(m) - 1) | (lane << 5) | (r << 11));
+        r = 0;
+        for (uint32_t m = nhi; m && off < r0 + kCap; m &= m - 1, r++, off++)
+            if (off >= r0) el[off - r0] = (uint16_t)((__ffs(m) - 1) | ((lane + 32) << 5) | (r << 11));
+        __syncwarp();
+        const uint32_t nr = min(etot - r0, kCap);
+        for (uint32_t p = lane; p < nr; p += 32) {
+            const uint32_t e = el[p];
+            const uint32_t src = e & 31u, t = (e >> 5) & 63u;
+            const uint32_t k = (uint32_t)((W.pk[0][src] >> t) & 1ull) | ((uint32_t)((W.pk[1][src] >> t) & 1ull) << 1) |
+                               ((uint32_t)((W.pk[2][src] >> t) & 1ull) << 2);
+            const size_t o = (size_t)(t + 64 * half) * P.n + sb[t] + (e >> 11);
+            P.qv[o] = W.iv[src];
+            P.parq[o] = W.li[k][src];
         }
+        __syncwarp();
     }
-    __syncwarp();
 }
 
 // parents of an item vertex whose whole adjacency fits one window (degree

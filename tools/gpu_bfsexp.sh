@@ -1,7 +1,6 @@
-timeout 900 python -m pytest tests -m gpu -x -q -k "randomized or stages or c3 or c4 or forest or given or hubs or degenerate" > gpurun_out/pytest_qrec.log 2>&1; echo pytest $?
-tail -3 gpurun_out/pytest_qrec.log
+timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_bfsexp.log 2>&1; echo pytest $?
+tail -3 gpurun_out/pytest_bfsexp.log
 run() { tag=$1; shift; timeout 300 python bench.py --no-cpu-baseline --no-e2e "$@" > gpurun_out/bench_$tag.log 2>&1; python -c "
 import json; d=json.loads(open('gpurun_out/bench_$tag.log').read().strip().splitlines()[-1]); print('$tag', round(d['value']/1e9,2), round(d['ms_per_step'],2), {k:round(v,2) for k,v in d['phase_ms_per_step'].items()})" || tail -3 gpurun_out/bench_$tag.log; }
-for c in c3 c4; do run ${c}_q0 --config $c; run ${c}_q1 --config $c --opt qrec=1; done
-run c3_q1s1 --opt qrec=1 --opt sub=1
-run c3_q1s2 --opt qrec=1 --opt sub=2
+for c in c3 c4 c2; do run ${c}_x --config $c; done
+run c5_x --config c5 --steps 2
