@@ -357,12 +357,21 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
     const uint32_t etot = __shfl_sync(0xFFFFFFFFu, eincl, 31);
     for (uint32_t r0 = 0; r0 < etot; r0 += kCap) {
         uint32_t off = eincl - ne;
-        uint32_t r = 0;
-        for (uint32_t m = nlo; m && off < r0 + kCap; m &= m - 1, r++, off++)
-            if (off >= r0) el[off - r0] = (uint16_t)((__ffs(m) - 1) | (lane << 5) | (r << 11));
-        r = 0;
-        for (uint32_t m = nhi; m && off < r0 + kCap; m &= m - 1, r++, off++)
-            if (off >= r0) el[off - r0] = (uint16_t)((__ffs(m) - 1) | ((lane + 32) << 5) | (r << 11));
+        if (etot <= kCap) {
+            // one round (the common case): no bounds to check
+            uint16_t *q = el + off;
+            uint32_t v = (lane << 5);
+            for (uint32_t m = nlo; m; m &= m - 1, v += 1u << 11) *q++ = (uint16_t)(v | (__ffs(m) - 1));
+            v = ((lane + 32) << 5);
+            for (uint32_t m = nhi; m; m &= m - 1, v += 1u << 11) *q++ = (uint16_t)(v | (__ffs(m) - 1));
+        } else {
+            uint32_t r = 0;
+            for (uint32_t m = nlo; m && off < r0 + kCap; m &= m - 1, r++, off++)
+                if (off >= r0) el[off - r0] = (uint16_t)((__ffs(m) - 1) | (lane << 5) | (r << 11));
+            r = 0;
+            for (uint32_t m = nhi; m && off < r0 + kCap; m &= m - 1, r++, off++)
+                if (off >= r0) el[off - r0] = (uint16_t)((__ffs(m) - 1) | ((lane + 32) << 5) | (r << 11));
+        }
         __syncwarp();
         const uint32_t nr = min(etot - r0, kCap);
         for (uint32_t p = lane; p < nr; p += 32) {
