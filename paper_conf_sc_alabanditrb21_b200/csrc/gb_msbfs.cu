@@ -299,16 +299,27 @@ __device__ __forceinline__ void ms_light_parents(const MsParams &P, const unsign
     const uint32_t total = __shfl_sync(0xFFFFFFFFu, incl, 31);
     for (uint32_t r0 = 0; r0 < total; r0 += kMultiCap) {
         uint32_t off = incl - cnt;
-        for (unsigned long long m = s2m; m; m &= m - 1) {
-            if (off >= r0 + kMultiCap) break;
-            if (off >= r0) {
+        if (total <= kMultiCap) {
+            // one round (the common case): no bounds to check
+            for (unsigned long long m = s2m; m; m &= m - 1) {
                 const int t = __ffsll((long long)m) - 1;
                 uint32_t km = 0;
 #pragma unroll
                 for (int k = 0; k < kLight; k++) km |= (uint32_t)((c[k] >> t) & 1ull) << k;
-                W.ml[off - r0] = ((uint32_t)lane << 14) | ((uint32_t)t << 8) | km;
+                W.ml[off++] = ((uint32_t)lane << 14) | ((uint32_t)t << 8) | km;
             }
-            off++;
+        } else {
+            for (unsigned long long m = s2m; m; m &= m - 1) {
+                if (off >= r0 + kMultiCap) break;
+                if (off >= r0) {
+                    const int t = __ffsll((long long)m) - 1;
+                    uint32_t km = 0;
+#pragma unroll
+                    for (int k = 0; k < kLight; k++) km |= (uint32_t)((c[k] >> t) & 1ull) << k;
+                    W.ml[off - r0] = ((uint32_t)lane << 14) | ((uint32_t)t << 8) | km;
+                }
+                off++;
+            }
         }
         __syncwarp();
         const uint32_t nr = min(total - r0, (uint32_t)kMultiCap);
@@ -428,10 +439,16 @@ __device__ __forceinline__ void ms_item_parents(const MsParams &P, const unsigne
     constexpr uint32_t kCap = 2 * kMultiCap;
     for (uint32_t r0 = 0; r0 < total; r0 += kCap) {
         uint32_t off = incl - cnt;
-        for (unsigned long long m = mm; m; m &= m - 1) {
-            if (off >= r0 + kCap) break;
-            if (off >= r0) pl[off - r0] = (uint16_t)((lane << 6) | (__ffsll((long long)m) - 1));
-            off++;
+        if (total <= kCap) {
+            // one round (the common case): no bounds to check
+            for (unsigned long long m = mm; m; m &= m - 1)
+                pl[off++] = (uint16_t)((lane << 6) | (__ffsll((long long)m) - 1));
+        } else {
+            for (unsigned long long m = mm; m; m &= m - 1) {
+                if (off >= r0 + kCap) break;
+                if (off >= r0) pl[off - r0] = (uint16_t)((lane << 6) | (__ffsll((long long)m) - 1));
+                off++;
+            }
         }
         __syncwarp();
         const uint32_t nr = min(total - r0, kCap);
