@@ -2,4 +2,4 @@ timeout 900 python -m pytest tests -m gpu -x -q -k "randomized or stages or c3 o
 tail -2 gpurun_out/pytest_bfsexp2.log
 run() { tag=$1; shift; timeout 300 python bench.py --no-cpu-baseline --no-e2e "$@" > gpurun_out/bench_$tag.log 2>&1; python -c "
 import json; d=json.loads(open('gpurun_out/bench_$tag.log').read().strip().splitlines()[-1]); print('$tag', round(d['value']/1e9,2), round(d['ms_per_step'],2), {k:round(v,2) for k,v in d['phase_ms_per_step'].items()})" || tail -3 gpurun_out/bench_$tag.log; }
-for c in c3 c4 c2; do run ${c}_z --config $c; done
+for c in c3 c4 c2; do run ${c}_d --config $c; done

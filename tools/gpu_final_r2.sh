@@ -6,7 +6,7 @@ python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/fin/smoke.log 2>
 timeout 900 python bench.py > gpurun_out/fin/bench_c3.json 2> gpurun_out/fin/bench_c3.err; echo c3 $?
 timeout 600 python bench.py --config c4 --steps 40 > gpurun_out/fin/bench_c4.json 2> gpurun_out/fin/bench_c4.err; echo c4 $?
 timeout 600 python bench.py --config c2 --steps 400 > gpurun_out/fin/bench_c2.json 2> gpurun_out/fin/bench_c2.err; echo c2 $?
-timeout 600 python bench.py --config c1 --steps 400 > gpurun_out/fin/bench_c1.json 2> gpurun_out/fin/bench_c1.err; echo c1 $?
+timeout 600 python bench.py --config c1 --steps 4000 > gpurun_out/fin/bench_c1.json 2> gpurun_out/fin/bench_c1.err; echo c1 $?
 timeout 900 python bench.py --config c5 --steps 3 --warmup 3 > gpurun_out/fin/bench_c5.json 2> gpurun_out/fin/bench_c5.err; echo c5 $?
 timeout 900 python bench.py --impl reference --steps 2 --warmup 3 > gpurun_out/fin/ref_c3.json 2> gpurun_out/fin/ref_c3.err; echo ref $?
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/fin/launches_c3.csv python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/fin/ncu_launch.log 2>&1; echo ncu $?
