@@ -76,6 +76,25 @@ __device__ __forceinline__ void warp_stats(int lane, int g, uint32_t k, bool cyc
     }
 }
 
+// the same from per-thread sums over many edges (one reduction per kernel)
+__device__ __forceinline__ void warp_stats_sum(int lane, int g, unsigned long long ks, uint32_t cs,
+                                               unsigned long long sig, unsigned long long *s_k,
+                                               unsigned long long *s_c, unsigned long long *s_sig) {
+#pragma unroll
+    for (int d = 16; d; d >>= 1) {
+        ks += __shfl_xor_sync(0xFFFFFFFFu, ks, d);
+        cs += __shfl_xor_sync(0xFFFFFFFFu, cs, d);
+        sig ^= __shfl_xor_sync(0xFFFFFFFFu, sig, d);
+    }
+    if (lane == 0) {
+        if (cs) {
+            atomicAdd(&s_k[g], ks);
+            atomicAdd(&s_c[g], (unsigned long long)cs);
+        }
+        if (sig) atomicXor(&s_sig[g], sig);
+    }
+}
+
 __device__ __forceinline__ void flush_stats(const CycleParams &P, const unsigned long long *s_k,
                                             const unsigned long long *s_c,
                                             const unsigned long long *s_sig) {
@@ -222,30 +241,32 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_pclimb(CycleParams P) {
 // test is on the parent words, and a climb step is one 16-byte gather; the
 // ancestors the climbs share (hubs and other high-degree vertices, internal
 // ids at the front) sit in a dense, L2-hot region.
-__global__ void __launch_bounds__(kCycleBlock) k_cycles_irec(CycleParams P) {
+__global__ void __launch_bounds__(kCycleBlock, 8) k_cycles_irec(CycleParams P) {
     __shared__ unsigned long long s_k[kMaxGroup], s_c[kMaxGroup], s_sig[kMaxGroup];
     for (int i = threadIdx.x; i < P.G; i += blockDim.x) { s_k[i] = 0; s_c[i] = 0; s_sig[i] = 0; }
     __syncthreads();
     const int lane = threadIdx.x & 31;
     const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t word = gw; word < P.words; word += nw) {
-        const int64_t e = word * 32 + lane;
-        const bool valid = e < P.m;
-        uint2 ed = valid ? __ldg(P.edges + e) : make_uint2(0, 0);
-        const uint32_t u = ed.x, v = ed.y & kIdMask, nege = ed.y >> 31;
-        for (int g = 0; g < P.G; g++) {
-            const uint4 *rec = P.irec + (size_t)(P.b0 + g) * P.n;
-            uint32_t flip = 0, k = 0;
-            bool cyc = false;
-            if (valid) {
+    // tree by tree (the G trees of a cycle group re-read the edge list from
+    // L2); a tree's cycle statistics are summed per thread and reduced across
+    // the warp once, not per 32-edge word
+    for (int g = 0; g < P.G; g++) {
+        const uint4 *rec = P.irec + (size_t)(P.b0 + g) * P.n;
+        uint32_t *fb = P.fbits + (size_t)(P.b0 + g) * P.words;
+        unsigned long long a_k = 0, a_sig = 0;
+        uint32_t a_c = 0;
+        for (int64_t word = gw; word < P.words; word += nw) {
+            const int64_t e = word * 32 + lane;
+            uint32_t flip = 0;
+            if (e < P.m) {
+                const uint2 ed = __ldg(P.edges + e);
+                const uint32_t u = ed.x, v = ed.y & kIdMask;
                 uint4 rx = __ldg(rec_at(rec, u)), ry = __ldg(rec_at(rec, v));
                 // tree edge iff one endpoint is the other's parent (simple graph)
                 if ((rx.x & kIdMask) != v && (ry.x & kIdMask) != u) {
-                    cyc = true;
                     const uint32_t px = rx.y & kIdMask, py = ry.y & kIdMask;
-                    uint32_t c = 0;
-                    k = 1;
+                    uint32_t c = 0, k = 1;
                     bool ax = is_anc(px, rx.z, py), ay = is_anc(py, ry.z, px);
                     while (!(ax && ay)) {
                         if (!ax) {
@@ -261,13 +282,16 @@ __global__ void __launch_bounds__(kCycleBlock) k_cycles_irec(CycleParams P) {
                             ay = is_anc(ry.y & kIdMask, ry.z, px);
                         }
                     }
-                    flip = (c >> 31) ^ nege;
+                    flip = (c >> 31) ^ (ed.y >> 31);
+                    a_k += k;
+                    a_c++;
+                    if (flip) a_sig ^= mix64((uint64_t)e ^ kSigSalt);
                 }
             }
             const uint32_t bits = __ballot_sync(0xFFFFFFFFu, flip != 0);
-            if (lane == 0) P.fbits[(size_t)(P.b0 + g) * P.words + word] = bits;
-            warp_stats(lane, g, k, cyc, flip != 0, e, s_k, s_c, s_sig);
+            if (lane == 0) fb[word] = bits;
         }
+        warp_stats_sum(lane, g, a_k, a_c, a_sig, s_k, s_c, s_sig);
     }
     __syncthreads();
     flush_stats(P, s_k, s_c, s_sig);
