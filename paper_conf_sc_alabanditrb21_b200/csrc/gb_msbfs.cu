@@ -713,6 +713,9 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
         }
         MS_PROF(0);
         // ---------------- phase A: discoveries --------------------------------
+        // per-lane discovery counts of trees lane, lane + 32, lane + 64, lane + 96
+        // (summed over the warp's tiles, added to the block's table once)
+        uint32_t a_cnt0 = 0, a_cnt1 = 0, a_cnt2 = 0, a_cnt3 = 0;
         for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
             if (tile < nit_tiles) {
                 const int64_t k = tile * kMsWarps + wid;
@@ -744,10 +747,10 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                                 atomicAdd(&s_ff, 1u);
                             }
                         }
-                        if ((part.a >> lane) & 1ull) atomicAdd(&s_cnt[lane], 1u);
-                        if ((part.a >> (lane + 32)) & 1ull) atomicAdd(&s_cnt[lane + 32], 1u);
-                        if ((part.b >> lane) & 1ull) atomicAdd(&s_cnt[lane + 64], 1u);
-                        if ((part.b >> (lane + 32)) & 1ull) atomicAdd(&s_cnt[lane + 96], 1u);
+                        a_cnt0 += (uint32_t)(part.a >> lane) & 1u;
+                        a_cnt1 += (uint32_t)(part.a >> (lane + 32)) & 1u;
+                        a_cnt2 += (uint32_t)(part.b >> lane) & 1u;
+                        a_cnt3 += (uint32_t)(part.b >> (lane + 32)) & 1u;
                         if (lane == 0) atomicAdd(&s_fc, 1u);
                     }
                 }
@@ -786,13 +789,13 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                     // so that lane t counts trees t, t + 32, t + 64, t + 96
                     const uint32_t c0 = __popc(transpose32((uint32_t)nw.a));
                     const uint32_t c1 = __popc(transpose32((uint32_t)(nw.a >> 32)));
-                    if (c0) atomicAdd(&s_cnt[lane], c0);
-                    if (c1) atomicAdd(&s_cnt[lane + 32], c1);
+                    a_cnt0 += c0;
+                    a_cnt1 += c1;
                     if (__any_sync(0xFFFFFFFFu, nw.b != 0)) {
                         const uint32_t c2 = __popc(transpose32((uint32_t)nw.b));
                         const uint32_t c3 = __popc(transpose32((uint32_t)(nw.b >> 32)));
-                        if (c2) atomicAdd(&s_cnt[lane + 64], c2);
-                        if (c3) atomicAdd(&s_cnt[lane + 96], c3);
+                        a_cnt2 += c2;
+                        a_cnt3 += c3;
                     }
                 }
                 const uint32_t nf = __ballot_sync(0xFFFFFFFFu, nowfull);
@@ -809,6 +812,10 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                 }
             }
         }
+        if (a_cnt0) atomicAdd(&s_cnt[lane], a_cnt0);
+        if (a_cnt1) atomicAdd(&s_cnt[lane + 32], a_cnt1);
+        if (a_cnt2) atomicAdd(&s_cnt[lane + 64], a_cnt2);
+        if (a_cnt3) atomicAdd(&s_cnt[lane + 96], a_cnt3);
         __syncthreads();
         if (tid < kMsBatch) {
             P.mscnt[(size_t)tid * kMsMaxBlocks + blockIdx.x] = s_cnt[tid];
