@@ -61,6 +61,7 @@ struct Options {
     int64_t wilson = 0;      // sampler 1: 0 one thread per tree (W trees at once), 1 parallel cycle popping
     int64_t harary = 0;      // 1: Harary sides by the L224 procedure (gb_harary.cu)
     int64_t jump = 1;        // walk 0: levels per ancestor record of the cycle walk (1, 2, 4)
+    int64_t push_parent = 1; // BFS, batches of <= 16 trees: parents chosen while pushing small frontiers
 };
 
 struct Stats {
@@ -112,7 +113,7 @@ static void free_ws(Workspace &w) {
                     w.parq, w.offq, w.szq, w.pp, w.rec, w.irec, w.prec, w.fbits, w.s1, w.tkey, w.depth,
                     w.tstat, w.visited, w.maxd, w.cidxq, w.cstart, w.clist, w.crec,
                     w.scan_tmp, w.vis, w.fr, w.hacc, w.hbest, w.msflag, w.mscnt, w.fbm, w.msprof,
-                    w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey,
+                    w.jrec, w.hlab, w.wbuf, w.wparent, w.wseq, w.wtkey, w.pnew, w.pbest,
                     w.ptbase, w.ptnbr, w.ptrng};
     for (void *p : ptrs) if (p) cudaFree(p);
     w = Workspace();
@@ -360,6 +361,7 @@ static int balance_range(int64_t t_begin, int64_t t_end, int64_t stride, uint64_
     // walk 1 keeps child lists of a whole batch in one 32-bit index space
     if (descent) B = (int)std::min<int64_t>(B, std::max<int64_t>(1, ((1ll << 32) - 1) / S.g.n));
     int rc = ensure_workspace(B, descent);
+    S.ws.pp_ok = S.opt.push_parent != 0;
     if (rc) return rc;
     const int G = auto_group(B);
     const int jump = S.opt.walk == 0 ? (int)S.opt.jump : 1;
@@ -663,6 +665,7 @@ int gb_set_option(const char *key, int64_t value) {
         if (value != 1 && value != 2 && value != 4) { set_error("walk_ept must be 1, 2 or 4"); return GB_EINVAL; }
         S.opt.walk_ept = value;
     }
+    else if (!strcmp(key, "push_parent")) S.opt.push_parent = value != 0;
     else if (!strcmp(key, "timing")) S.opt.timing = value != 0;
     else if (!strcmp(key, "sub")) { if (value < 0) return GB_EINVAL; S.opt.sub = value; }
     else if (!strcmp(key, "msprof")) S.opt.msprof = value != 0;

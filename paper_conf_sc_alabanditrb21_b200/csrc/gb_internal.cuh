@@ -187,6 +187,10 @@ struct Workspace {
                                         // [4..6] frontier sizes (levels mod 3)
     uint32_t *mscnt = nullptr;          // [128][2048] per-block discovery counts
     unsigned long long *msprof = nullptr;  // [256][4] BFS phase timestamps (option "msprof")
+    unsigned long long *pnew = nullptr;    // push-parent levels (<= 16 trees): [n] discoveries
+    unsigned long long *pbest = nullptr;   // [n][16] best parent keys (all ones between uses)
+    bool pp_ok = true;                     // option "push_parent"
+    bool pp_nomem = false;                 // not enough free memory for the push-parent state
     uint32_t *fbm = nullptr;            // [6][ceil(n/32)] frontier bitmaps (3), finished bitmap,
                                         // two push bitmaps (direction optimisation)
     uint32_t *s1 = nullptr;    // [B][ncomp] #vertices with pi = 1 per component

@@ -40,6 +40,7 @@ namespace gb {
 namespace cg = cooperative_groups;
 
 constexpr int kMsMaxBlocks = 2048;   // capacity of the per-block count table
+constexpr int kPPTrees = 16;         // push-parent levels: batches of <= 16 trees
 
 struct MsParams {
     const uint32_t *brow, *badj, *borig, *bord, *brank;
@@ -56,6 +57,8 @@ struct MsParams {
     uint32_t *fcnt;    // [3] vertices on the frontier of level L (mod 3); [3] vertices finished
     int64_t push_div;  // a level pushes first while frontier * push_div <= unfinished vertices
     int32_t *flag;
+    unsigned long long *pnew;   // push-parent levels: [n] trees discovering the vertex (or null)
+    unsigned long long *pbest;  // push-parent levels: [n][kPPTrees] best parent keys (~0 = none)
     uint32_t *mscnt;   // [128][kMsMaxBlocks] discoveries per tree per block (phase A)
     const uint64_t *tkey;
     uint32_t *qv, *parq, *pp;
@@ -613,6 +616,31 @@ __global__ void k_ms_roots(MsParams P) {
     }
 }
 
+// push-parent levels: candidate (u -> x) of the frontier vertex u (trees fu,
+// original id ou) through adjacency slot j (a = badj[j])
+__device__ __forceinline__ void pp_push(const MsParams &P, unsigned long long fu, uint32_t ou,
+                                        uint32_t a, uint32_t j, const uint64_t *s_tk) {
+    const uint32_t x = a & kIdMask;
+    const unsigned long long want = fu & ~__ldcg(P.vis + x);
+    if (!want) return;
+    atomicOr(P.pnew + x, want);
+    const uint32_t ox = __ldg(P.borig + j);
+    for (unsigned long long m = want; m; m &= m - 1) {
+        const int t = __ffsll((long long)m) - 1;
+        atomicMin(P.pbest + (size_t)x * kPPTrees + t, parent_key(s_tk[t], ou, ox, a >> 31));
+    }
+}
+
+// push-parent levels: the entry of vertex i in tree t (its best key, then the
+// slot is reset for the next use)
+__device__ __forceinline__ void pp_emit(const MsParams &P, int t, uint32_t i, const uint32_t *s_base,
+                                        uint32_t *s_pos) {
+    unsigned long long *slot = P.pbest + (size_t)i * kPPTrees + t;
+    const unsigned long long key = __ldcg(slot);
+    *slot = ~0ull;
+    ms_emit(P, t, s_base[t] + atomicAdd(&s_pos[t], 1u), i, key);
+}
+
 // ---------------------------------------------------------------------------
 // the BFS: one cooperative kernel.  Per level L:
 //   phase A  every block pulls over its tiles (static: tile k -> block
@@ -687,15 +715,26 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                                    : __ldcg(P.fcnt + L % 3);
         const int64_t unfinished = P.n - (int64_t)__ldcg(P.fcnt + 3);
         const bool push = (int64_t)fc * P.push_div <= unfinished;
+        // Push-parent levels (batches of <= 16 trees): the push itself
+        // discovers -- new(x) |= F_L(u) & ~vis(x) -- and selects the parents:
+        // every (frontier vertex u, neighbour x, tree t) candidate takes part
+        // in an atomicMin of parent_key(t, u, x) (reading R4: the same
+        // minimum over the same candidates), so phases A and B read one word
+        // per marked vertex instead of scanning its adjacency (on RMAT the
+        // marked hubs hold millions of slots)
+        const bool pp = S == 1 && push && P.pbest != nullptr && B <= kPPTrees;
         uint32_t *tbc = P.tb + (size_t)(L & 1) * P.nwords;
         if (push) {
             for (int64_t k = gwarp; k < P.nitems; k += nwarps) {
                 const uint2 it = __ldg(P.items + k);
                 if (!bm_test(bm, it.x)) continue;
                 const uint32_t s1 = min(it.y + (uint32_t)kChunk, __ldg(P.brow + it.x + 1));
+                const unsigned long long fu = pp ? __ldcg(F + it.x) : 0ull;
+                const uint32_t ou = pp ? __ldg(P.bord + it.x) : 0u;
                 for (uint32_t j = it.y + lane; j < s1; j += 32) {
-                    const uint32_t x = __ldg(P.badj + j) & kIdMask;
+                    const uint32_t a = __ldg(P.badj + j), x = a & kIdMask;
                     atomicOr(tbc + (x >> 5), 1u << (x & 31));
+                    if (pp) pp_push(P, fu, ou, a, j, s_tk);
                 }
             }
             for (int64_t w = (P.nlight0 >> 5) + gwarp; w < P.nwords; w += nwarps) {
@@ -704,9 +743,12 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                 if (!((word >> lane) & 1u)) continue;
                 const uint32_t u = (uint32_t)(w * 32 + lane);
                 const uint32_t rs = __ldg(P.brow + u), re = __ldg(P.brow + u + 1);
+                const unsigned long long fu = pp ? __ldcg(F + u) : 0ull;
+                const uint32_t ou = pp ? __ldg(P.bord + u) : 0u;
                 for (uint32_t j = rs; j < re; j++) {
-                    const uint32_t x = __ldg(P.badj + j) & kIdMask;
+                    const uint32_t a = __ldg(P.badj + j), x = a & kIdMask;
                     atomicOr(tbc + (x >> 5), 1u << (x & 31));
+                    if (pp) pp_push(P, fu, ou, a, j, s_tk);
                 }
             }
             grid.sync();
@@ -724,10 +766,18 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                     const uint32_t i = it.x, s0 = it.y;
                     if (bm_test(P.fullbm, i)) continue;
                     if (push && !bm_test(tbc, i)) continue;
+                    if (pp && s0 != __ldg(P.brow + i)) continue;   // the vertex's first chunk stands for it
                     const uint32_t s1 = min(s0 + (uint32_t)kChunk, __ldg(P.brow + i + 1));
-                    const bool multi = k < P.nmulti_items;
+                    const bool multi = !pp && k < P.nmulti_items;
                     const W2 vis = ld2<S>(P.vis + S * (size_t)i);
-                    W2 part = ms_chunk_or<S>(P, F, bm, s0, s1);
+                    W2 part;
+                    if (pp) {
+                        part = W2{__ldcg(P.pnew + i), 0ull};
+                        __syncwarp();
+                        if (lane == 0 && part.a) P.pnew[i] = 0ull;
+                    } else {
+                        part = ms_chunk_or<S>(P, F, bm, s0, s1);
+                    }
                     part.a &= ~vis.a;
                     part.b &= ~vis.b;
                     if (multi) {
@@ -768,13 +818,18 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                     const uint32_t rs = __ldg(P.brow + i);
                     const uint32_t deg = __ldg(P.brow + i + 1) - rs;
                     W2 acc{0ull, 0ull};
+                    if (pp) {
+                        acc.a = __ldcg(P.pnew + i);
+                        if (acc.a) P.pnew[i] = 0ull;
+                    } else {
 #pragma unroll
-                    for (int k = 0; k < kLight; k++)
-                        if (k < (int)deg) {
-                            const W2 w = fr_word2<S>(F, bm, __ldg(P.badj + rs + k) & kIdMask);
-                            acc.a |= w.a;
-                            acc.b |= w.b;
-                        }
+                        for (int k = 0; k < kLight; k++)
+                            if (k < (int)deg) {
+                                const W2 w = fr_word2<S>(F, bm, __ldg(P.badj + rs + k) & kIdMask);
+                                acc.a |= w.a;
+                                acc.b |= w.b;
+                            }
+                    }
                     nw = W2{acc.a & ~vis.a, acc.b & ~vis.b};
                     const W2 nv{vis.a | nw.a, vis.b | nw.b};
                     if (nw.a | nw.b) {
@@ -860,7 +915,13 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
         for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
             if (tile < nit_tiles) {
                 const int64_t k = tile * kMsWarps + wid;
-                if (k < P.nitems && k >= P.nmulti_items) {
+                if (pp && k < P.nitems) {
+                    const uint2 it = __ldg(P.items + k);
+                    const uint32_t i = it.x;
+                    if (it.y != __ldg(P.brow + i) || !bm_test(nbm, i)) continue;
+                    const unsigned long long nw = __ldcg(Nx + i);
+                    if (lane < B && ((nw >> lane) & 1ull)) pp_emit(P, lane, i, s_base, s_pos);
+                } else if (k < P.nitems && k >= P.nmulti_items) {
                     const uint2 it = __ldg(P.items + k);
                     const uint32_t i = it.x;
                     if (!bm_test(nbm, i)) continue;
@@ -895,6 +956,14 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                 uint32_t fb = __ldcg(nbm + (v0 >> 5));
                 if (v0 < P.nlight0) fb &= ~0u << (uint32_t)(P.nlight0 - v0);   // item lanes are not ours
                 if (!fb) continue;
+                if (pp) {
+                    if ((fb >> lane) & 1u) {
+                        const uint32_t i = (uint32_t)(v0 + lane);
+                        for (unsigned long long m = __ldcg(Nx + i); m; m &= m - 1)
+                            pp_emit(P, __ffsll((long long)m) - 1, i, s_base, s_pos);
+                    }
+                    continue;
+                }
                 if ((fb >> lane) & 1u) s_q[wid][qn + __popc(fb & ((1u << lane) - 1u))] = (uint32_t)(v0 + lane);
                 qn += __popc(fb);
                 if (qn >= 32) {
@@ -1034,6 +1103,24 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
     P.fcnt = reinterpret_cast<uint32_t *>(ws.msflag + 4);
     P.push_div = 32;   // measured on C3: 32 and 128 equal (bfs 59.0 ms / 100 trees), 8 worse (61.3)
     P.flag = ws.msflag; P.mscnt = ws.mscnt;
+    P.pnew = nullptr; P.pbest = nullptr;
+    if (S == 1 && B <= kPPTrees && ws.pp_ok && !ws.pp_nomem) {
+        // push-parent state, allocated once (all-zero / all-ones between uses)
+        if (!ws.pbest) {
+            size_t fr = 0, tot = 0;
+            const size_t need = sizeof(unsigned long long) * (size_t)g.n * (kPPTrees + 1);
+            if (cudaMemGetInfo(&fr, &tot) == cudaSuccess && fr > 2 * need) {
+                GB_CUDA_TRY(cudaMalloc(&ws.pnew, sizeof(unsigned long long) * (size_t)g.n));
+                GB_CUDA_TRY(cudaMalloc(&ws.pbest, sizeof(unsigned long long) * (size_t)g.n * kPPTrees));
+                GB_CUDA_TRY(cudaMemsetAsync(ws.pnew, 0, sizeof(unsigned long long) * (size_t)g.n, st));
+                GB_CUDA_TRY(cudaMemsetAsync(ws.pbest, 0xFF, sizeof(unsigned long long) * (size_t)g.n * kPPTrees, st));
+            } else {
+                ws.pp_nomem = true;
+            }
+        }
+        P.pnew = ws.pnew;
+        P.pbest = ws.pbest;
+    }
     P.tkey = o.tkey; P.qv = o.qv; P.parq = o.parq; P.pp = o.pp; P.rec = o.rec; P.crec = o.crec; P.irec = o.irec; P.prec = o.prec;
     P.lvl = o.lvl; P.vbase = o.vbase; P.depth = o.depth; P.maxd = o.maxd;
     P.prof = ws.msprof;
