@@ -35,6 +35,7 @@
 #include "../../include/graphb.h"
 
 #include <algorithm>
+#include <cstdlib>
 
 namespace gb {
 namespace cg = cooperative_groups;
@@ -59,6 +60,7 @@ struct MsParams {
     int32_t *flag;
     unsigned long long *pnew;   // push-parent levels: [n] trees discovering the vertex (or null)
     unsigned long long *pbest;  // push-parent levels: [n][kPPTrees] best parent keys (~0 = none)
+    int pp_from;                // first level that may use them
     uint32_t *mscnt;   // [128][kMsMaxBlocks] discoveries per tree per block (phase A)
     const uint64_t *tkey;
     uint32_t *qv, *parq, *pp;
@@ -722,7 +724,7 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
         // minimum over the same candidates), so phases A and B read one word
         // per marked vertex instead of scanning its adjacency (on RMAT the
         // marked hubs hold millions of slots)
-        const bool pp = S == 1 && push && P.pbest != nullptr && B <= kPPTrees;
+        const bool pp = S == 1 && push && P.pbest != nullptr && B <= kPPTrees && L >= P.pp_from;
         uint32_t *tbc = P.tb + (size_t)(L & 1) * P.nwords;
         if (push) {
             for (int64_t k = gwarp; k < P.nitems; k += nwarps) {
@@ -1104,6 +1106,9 @@ int run_msbfs(const Graph &g, Workspace &ws, int B, const MsBfsOut &o, cudaStrea
     P.push_div = 32;   // measured on C3: 32 and 128 equal (bfs 59.0 ms / 100 trees), 8 worse (61.3)
     P.flag = ws.msflag; P.mscnt = ws.mscnt;
     P.pnew = nullptr; P.pbest = nullptr;
+    // level 0 pulls: its frontier is one root per tree in every component of
+    // >= 2 vertices (RMAT-26: ~10 M pushes), measured C5 bfs 242.6 vs 238.2 ms
+    P.pp_from = 1;
     if (S == 1 && B <= kPPTrees && ws.pp_ok && !ws.pp_nomem) {
         // push-parent state, allocated once (all-zero / all-ones between uses)
         if (!ws.pbest) {
