@@ -132,7 +132,10 @@ int gb_balance_given_tree(const int32_t *parent, uint8_t *flip,
  * cycle popping and processed one tree at a time; gb_tree_debug then reports
  * that tree; 2 = DFS trees with a hashed scan start per vertex, reading R18),
  * "wilson" (sampler 1: 0 = one GPU thread per tree, 1 = parallel cycle
- * popping), "reset" (every option back to its default). */
+ * popping), "push_parent" (1 = default: BFS batches of <= 16 trees choose the
+ * parents of small-frontier levels while pushing -- the same R4 minimum over
+ * the same candidates; 0 = always pull), "reset" (every option back to its
+ * default). */
 int gb_set_option(const char *key, int64_t value);
 
 /* Statistics of the last gb_balance / gb_balance_range call (waits for its

@@ -64,7 +64,7 @@ def test_state_and_argument_errors_without_gpu():
     assert L.gb_set_option(b"sampler", -1) == graphb.GB_EINVAL
     assert L.gb_set_option(b"jump", 3) == graphb.GB_EINVAL         # 1, 2 or 4 levels
     for k, v in [(b"sampler", 2), (b"wilson", 1), (b"harary", 1), (b"jump", 4), (b"recpass", 0),
-                 (b"walk", 2), (b"walk", 3), (b"desc_linear", 1), (b"walk_ept", 4),
+                 (b"walk", 2), (b"walk", 3), (b"desc_linear", 1), (b"walk_ept", 4), (b"push_parent", 0),
                  (b"batch", 128)]:
         assert L.gb_set_option(k, v) == 0
     assert L.gb_set_option(b"reset", 0) == 0

@@ -623,7 +623,7 @@ def _sweep_case(i):
     else:
         g = graphgen.rmat(int(rng.integers(7, 11)), 8, 0.3, 50 + i)
     T = int(rng.choice([1, 2, 31, 63, 64, 65, 100, 127, 128, 129, 140]))
-    opts = {"walk": int(rng.choice([0, 0, 3, 1, 2])),
+    opts = {"walk": int(rng.choice([0, 0, 3, 1, 2])), "push_parent": int(rng.integers(0, 2)),
             "batch": int(rng.choice([0, 0, 1, 7, 64, 65, 128])),
             "cycle_group": int(rng.choice([0, 1, 3])),
             "sub": int(rng.choice([0, 1, 3]))}
