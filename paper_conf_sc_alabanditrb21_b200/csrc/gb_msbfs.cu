@@ -716,7 +716,11 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
         const uint32_t fc = L == 0 ? (uint32_t)(((int64_t)B * P.nbig < P.n) ? (int64_t)B * P.nbig : P.n)
                                    : __ldcg(P.fcnt + L % 3);
         const int64_t unfinished = P.n - (int64_t)__ldcg(P.fcnt + 3);
-        const bool push = (int64_t)fc * P.push_div <= unfinished;
+        // batches that can take the push-parent path also push whenever the
+        // frontier is small against the whole graph (the last levels, where
+        // a pull still walks every tile for a few unfinished vertices)
+        const bool ppcap = S == 1 && P.pbest != nullptr && B <= kPPTrees && L >= P.pp_from;
+        const bool push = (int64_t)fc * P.push_div <= unfinished || (ppcap && (int64_t)fc * 64 <= P.n);
         // Push-parent levels (batches of <= 16 trees): the push itself
         // discovers -- new(x) |= F_L(u) & ~vis(x) -- and selects the parents:
         // every (frontier vertex u, neighbour x, tree t) candidate takes part
@@ -724,19 +728,27 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
         // minimum over the same candidates), so phases A and B read one word
         // per marked vertex instead of scanning its adjacency (on RMAT the
         // marked hubs hold millions of slots)
-        const bool pp = S == 1 && push && P.pbest != nullptr && B <= kPPTrees && L >= P.pp_from;
+        const bool pp = ppcap && push;
         uint32_t *tbc = P.tb + (size_t)(L & 1) * P.nwords;
         if (push) {
-            for (int64_t k = gwarp; k < P.nitems; k += nwarps) {
-                const uint2 it = __ldg(P.items + k);
-                if (!bm_test(bm, it.x)) continue;
-                const uint32_t s1 = min(it.y + (uint32_t)kChunk, __ldg(P.brow + it.x + 1));
-                const unsigned long long fu = pp ? __ldcg(F + it.x) : 0ull;
-                const uint32_t ou = pp ? __ldg(P.bord + it.x) : 0u;
-                for (uint32_t j = it.y + lane; j < s1; j += 32) {
-                    const uint32_t a = __ldg(P.badj + j), x = a & kIdMask;
-                    atomicOr(tbc + (x >> 5), 1u << (x & 31));
-                    if (pp) pp_push(P, fu, ou, a, j, s_tk);
+            // the work items of frontier vertices: a warp tests 32 items at a
+            // time and walks the chunks of those on the frontier
+            for (int64_t k0 = gwarp * 32; k0 < P.nitems; k0 += nwarps * 32) {
+                const int64_t kk = k0 + lane;
+                const uint2 itl = kk < P.nitems ? __ldg(P.items + kk) : make_uint2(0u, 0u);
+                for (uint32_t fm = __ballot_sync(0xFFFFFFFFu, kk < P.nitems && bm_test(bm, itl.x)); fm;
+                     fm &= fm - 1) {
+                    const int src = __ffs(fm) - 1;
+                    const uint2 it = make_uint2(__shfl_sync(0xFFFFFFFFu, itl.x, src),
+                                                __shfl_sync(0xFFFFFFFFu, itl.y, src));
+                    const uint32_t s1 = min(it.y + (uint32_t)kChunk, __ldg(P.brow + it.x + 1));
+                    const unsigned long long fu = pp ? __ldcg(F + it.x) : 0ull;
+                    const uint32_t ou = pp ? __ldg(P.bord + it.x) : 0u;
+                    for (uint32_t j = it.y + lane; j < s1; j += 32) {
+                        const uint32_t a = __ldg(P.badj + j), x = a & kIdMask;
+                        atomicOr(tbc + (x >> 5), 1u << (x & 31));
+                        if (pp) pp_push(P, fu, ou, a, j, s_tk);
+                    }
                 }
             }
             for (int64_t w = (P.nlight0 >> 5) + gwarp; w < P.nwords; w += nwarps) {
@@ -760,6 +772,41 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
         // per-lane discovery counts of trees lane, lane + 32, lane + 64, lane + 96
         // (summed over the warp's tiles, added to the block's table once)
         uint32_t a_cnt0 = 0, a_cnt1 = 0, a_cnt2 = 0, a_cnt3 = 0;
+        if (pp) {
+            // push-parent level: every marked vertex reads its discoveries
+            // from pnew; a warp owns whole 32-vertex words (the same static
+            // mapping in phase B), so no hub chunk or adjacency is visited
+            for (int64_t w = (int64_t)blockIdx.x * kMsWarps + wid; w < P.nwords;
+                 w += (int64_t)gridDim.x * kMsWarps) {
+                const uint32_t i = (uint32_t)(w * 32 + lane);
+                const uint32_t tw = __ldcg(tbc + w), fw = __ldcg(P.fullbm + w);
+                unsigned long long nwv = 0;
+                bool nowfull = false;
+                if ((int64_t)i < P.n && ((tw >> lane) & 1u) && !((fw >> lane) & 1u)) {
+                    const unsigned long long pn = __ldcg(P.pnew + i);
+                    if (pn) {
+                        P.pnew[i] = 0ull;
+                        const unsigned long long vis = __ldcg(P.vis + S * (size_t)i);
+                        nwv = pn & ~vis;
+                        if (nwv) {
+                            const unsigned long long nv = vis | nwv;
+                            P.vis[S * (size_t)i] = nv;
+                            Nx[S * (size_t)i] = nwv;
+                            nowfull = nv == full.a;
+                        }
+                    }
+                }
+                const uint32_t fb = __ballot_sync(0xFFFFFFFFu, nwv != 0);
+                if (fb) a_cnt0 += __popc(transpose32((uint32_t)nwv));   // <= 16 trees
+                const uint32_t nf = __ballot_sync(0xFFFFFFFFu, nowfull);
+                if (lane == 0) {
+                    if (fb) atomicAdd(&s_fc, (uint32_t)__popc(fb));
+                    if (nf) atomicAdd(&s_ff, (uint32_t)__popc(nf));
+                    nbm[w] = fb;
+                    if (nf) P.fullbm[w] = fw | nf;
+                }
+            }
+        } else
         for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
             if (tile < nit_tiles) {
                 const int64_t k = tile * kMsWarps + wid;
@@ -768,18 +815,10 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                     const uint32_t i = it.x, s0 = it.y;
                     if (bm_test(P.fullbm, i)) continue;
                     if (push && !bm_test(tbc, i)) continue;
-                    if (pp && s0 != __ldg(P.brow + i)) continue;   // the vertex's first chunk stands for it
                     const uint32_t s1 = min(s0 + (uint32_t)kChunk, __ldg(P.brow + i + 1));
-                    const bool multi = !pp && k < P.nmulti_items;
+                    const bool multi = k < P.nmulti_items;
                     const W2 vis = ld2<S>(P.vis + S * (size_t)i);
-                    W2 part;
-                    if (pp) {
-                        part = W2{__ldcg(P.pnew + i), 0ull};
-                        __syncwarp();
-                        if (lane == 0 && part.a) P.pnew[i] = 0ull;
-                    } else {
-                        part = ms_chunk_or<S>(P, F, bm, s0, s1);
-                    }
+                    W2 part = ms_chunk_or<S>(P, F, bm, s0, s1);
                     part.a &= ~vis.a;
                     part.b &= ~vis.b;
                     if (multi) {
@@ -820,18 +859,13 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                     const uint32_t rs = __ldg(P.brow + i);
                     const uint32_t deg = __ldg(P.brow + i + 1) - rs;
                     W2 acc{0ull, 0ull};
-                    if (pp) {
-                        acc.a = __ldcg(P.pnew + i);
-                        if (acc.a) P.pnew[i] = 0ull;
-                    } else {
 #pragma unroll
-                        for (int k = 0; k < kLight; k++)
-                            if (k < (int)deg) {
-                                const W2 w = fr_word2<S>(F, bm, __ldg(P.badj + rs + k) & kIdMask);
-                                acc.a |= w.a;
-                                acc.b |= w.b;
-                            }
-                    }
+                    for (int k = 0; k < kLight; k++)
+                        if (k < (int)deg) {
+                            const W2 w = fr_word2<S>(F, bm, __ldg(P.badj + rs + k) & kIdMask);
+                            acc.a |= w.a;
+                            acc.b |= w.b;
+                        }
                     nw = W2{acc.a & ~vis.a, acc.b & ~vis.b};
                     const W2 nv{vis.a | nw.a, vis.b | nw.b};
                     if (nw.a | nw.b) {
@@ -914,16 +948,21 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
             }
         }
         __syncthreads();
+        if (pp) {
+            for (int64_t w = (int64_t)blockIdx.x * kMsWarps + wid; w < P.nwords;
+                 w += (int64_t)gridDim.x * kMsWarps) {
+                const uint32_t fb = __ldcg(nbm + w);
+                if ((fb >> lane) & 1u) {
+                    const uint32_t i = (uint32_t)(w * 32 + lane);
+                    for (unsigned long long m = __ldcg(Nx + S * (size_t)i); m; m &= m - 1)
+                        pp_emit(P, __ffsll((long long)m) - 1, i, s_base, s_pos);
+                }
+            }
+        } else
         for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
             if (tile < nit_tiles) {
                 const int64_t k = tile * kMsWarps + wid;
-                if (pp && k < P.nitems) {
-                    const uint2 it = __ldg(P.items + k);
-                    const uint32_t i = it.x;
-                    if (it.y != __ldg(P.brow + i) || !bm_test(nbm, i)) continue;
-                    const unsigned long long nw = __ldcg(Nx + i);
-                    if (lane < B && ((nw >> lane) & 1ull)) pp_emit(P, lane, i, s_base, s_pos);
-                } else if (k < P.nitems && k >= P.nmulti_items) {
+                if (k < P.nitems && k >= P.nmulti_items) {
                     const uint2 it = __ldg(P.items + k);
                     const uint32_t i = it.x;
                     if (!bm_test(nbm, i)) continue;
@@ -958,14 +997,6 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
                 uint32_t fb = __ldcg(nbm + (v0 >> 5));
                 if (v0 < P.nlight0) fb &= ~0u << (uint32_t)(P.nlight0 - v0);   // item lanes are not ours
                 if (!fb) continue;
-                if (pp) {
-                    if ((fb >> lane) & 1u) {
-                        const uint32_t i = (uint32_t)(v0 + lane);
-                        for (unsigned long long m = __ldcg(Nx + i); m; m &= m - 1)
-                            pp_emit(P, __ffsll((long long)m) - 1, i, s_base, s_pos);
-                    }
-                    continue;
-                }
                 if ((fb >> lane) & 1u) s_q[wid][qn + __popc(fb & ((1u << lane) - 1u))] = (uint32_t)(v0 + lane);
                 qn += __popc(fb);
                 if (qn >= 32) {
