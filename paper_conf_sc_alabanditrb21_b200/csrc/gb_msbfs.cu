@@ -42,6 +42,9 @@ namespace cg = cooperative_groups;
 
 constexpr int kMsMaxBlocks = 2048;   // capacity of the per-block count table
 constexpr int kPPTrees = 16;         // push-parent levels: batches of <= 16 trees
+#ifndef GB_PP_DIV
+#define GB_PP_DIV 64
+#endif
 
 struct MsParams {
     const uint32_t *brow, *badj, *borig, *bord, *brank;
@@ -720,7 +723,7 @@ __global__ void __launch_bounds__(kBlock, GB_MS_MINBLOCKS) k_msbfs(MsParams P) {
         // frontier is small against the whole graph (the last levels, where
         // a pull still walks every tile for a few unfinished vertices)
         const bool ppcap = S == 1 && P.pbest != nullptr && B <= kPPTrees && L >= P.pp_from;
-        const bool push = (int64_t)fc * P.push_div <= unfinished || (ppcap && (int64_t)fc * 64 <= P.n);
+        const bool push = (int64_t)fc * P.push_div <= unfinished || (ppcap && (int64_t)fc * GB_PP_DIV <= P.n);
         // Push-parent levels (batches of <= 16 trees): the push itself
         // discovers -- new(x) |= F_L(u) & ~vis(x) -- and selects the parents:
         // every (frontier vertex u, neighbour x, tree t) candidate takes part
